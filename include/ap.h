@@ -1,0 +1,236 @@
+/*
+ * ap.h -- C ABI of the B200-native AutoPipe planner/slicer hot path.
+ *
+ * The library (paper_conf_cluster_liulldgl22_b200/libap.so, sm_100a) simulates
+ * candidate pipeline partitions under the 1F1B schedule and searches them.  Every
+ * step of the path runs in CUDA kernels; the host code only validates, allocates
+ * and launches.  No exceptions and no torch types cross this boundary.
+ *
+ * Citations: "PAPER.md:N" is line N of the AutoPipe paper text (Liu et al., IEEE
+ * CLUSTER 2022) with the section/equation/algorithm it belongs to; DESIGN.md
+ * readings Q1..Q26 fix what the paper leaves open.
+ *
+ * Conventions for every call:
+ *  - Times are int64 nanoseconds.  Results are bit-exact with the CPU oracle.
+ *  - Sub-layer i in [0,n) is one block of the model (Fig. 3: embedding,
+ *    ResidualAttentionBlock / ResidualFFNBlock halves of each layer, head).
+ *  - A partition of n sub-layers into p stages is its cut vector
+ *    cuts[0..p-2] = (c_1 < ... < c_{p-1}), every c in [1, n-1]; stage x owns
+ *    sub-layers [c_x, c_{x+1}) with c_0 = 0, c_p = n.
+ *    Partitions are ranked in lexicographic order of their cut vectors.
+ *  - Ownership: the plan owns its device tables.  The caller owns every buffer it
+ *    passes.  Device pointers must be on the plan's device.
+ *  - Synchronisation: calls that write device outputs are asynchronous and
+ *    stream-ordered on `stream` (ap_eval_batch, ap_search_*), except that
+ *    ap_search_* synchronise once on `stream` to read the reference time T_ref.
+ *    Calls with host outputs block until they are ready.
+ *  - Errors: every call returns an ap_status.  The message of the most recent
+ *    failure on the calling thread is available from ap_last_error().  On error
+ *    the outputs are unspecified.  A missing/unsupported GPU is AP_ERR_CUDA: there
+ *    is no CPU fallback.
+ *  - Thread safety: a plan is immutable after creation; concurrent calls on
+ *    different streams are safe.
+ */
+#ifndef AP_H_
+#define AP_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* ap_stream_t; /* == cudaStream_t; NULL = legacy default */
+
+#define AP_MAX_P 32   /* pipeline stages  */
+#define AP_MAX_K 16   /* slice pieces of micro-batch 0 */
+#define AP_MAX_N 512  /* sub-layers       */
+
+typedef enum {
+  AP_OK = 0,
+  AP_ERR_INVALID = 1,  /* argument out of its documented domain          */
+  AP_ERR_RANGE = 2,    /* int64 overflow guard or 63-bit key packing      */
+  AP_ERR_CUDA = 3,     /* CUDA runtime error / no sm_100 device           */
+  AP_ERR_NOMEM = 4,    /* device or host allocation failed                */
+  AP_ERR_CAPACITY = 5  /* caller buffer too small                         */
+} ap_status;
+
+/* Message describing the last failure on this thread ("" if none). */
+const char* ap_last_error(void);
+
+/* Library version string and the compute capability it was built for. */
+const char* ap_version(void);
+
+typedef struct ap_plan ap_plan; /* opaque, immutable after create */
+
+/*
+ * ap_plan_create -- stage the model's profiled costs on `device`.
+ * PAPER.md:81 (§III-A "model configs ... runtime statistics"), Alg. 1 line 1
+ * ("Get forward time f_i and backward time b_i for block i").
+ *   n                 number of sub-layers, 1 <= n <= AP_MAX_N
+ *   fwd_ns, bwd_ns    host int64[n], >= 0: forward / backward time of sub-layer i
+ *   act_bytes         host int64[n], >= 0: bytes of the activation leaving sub-layer
+ *                     i (= the gradient entering it); entry n-1 is ignored
+ *   link_bytes_per_s  > 0.  comm_ns[i] = ceil(act_bytes[i]*1e9 / link), 128-bit
+ *                     exact ("Comm"; BASELINE north_star "activation
+ *                     bytes over link bandwidth"; reading Q4/Q25)
+ *   device            CUDA ordinal; must be an sm_100 (B200) device
+ *   out               receives the plan
+ * Copies the tables host->device once (blocking).  Errors: INVALID, RANGE (a sum
+ * that cannot be held in int64), CUDA, NOMEM.
+ */
+ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns,
+                         const int64_t* act_bytes, uint64_t link_bytes_per_s,
+                         int32_t device, ap_plan** out);
+
+/* Release a plan and its device memory.  NULL-safe.  Not concurrent-safe with
+ * calls still running on the plan. */
+void ap_plan_destroy(ap_plan* plan);
+
+/* Number of sub-layers and comm_ns table (host copy) of a plan.  comm may be NULL. */
+ap_status ap_plan_info(const ap_plan* plan, int32_t* n, int64_t* comm_ns);
+
+/* C(n-1, p-1): the size of the partition space.  RANGE when it
+ * is >= 2^63.  INVALID unless 1 <= p <= n. */
+ap_status ap_count(int32_t n, int32_t p, uint64_t* out);
+
+/*
+ * ap_eval_batch -- iteration time (and master stage) of `count` candidates.
+ * The pipeline simulator of PAPER.md:103-125 (§III-B-1): 1F1B with m micro-batches
+ * (warm-up simulated exactly, reading Q1), Comm charged on the receiving stage
+ * (PAPER.md:115, :123), micro-batch 0's forward split into k pieces
+ * (PAPER.md:202-204 Slicer; BASELINE north_star).  T = end of the last backward of
+ * stage 0.  master = stage most visited by the unique critical path
+ * in the 1F1B phase (readings Q10, Q11).
+ *   p in [1, min(n, AP_MAX_P)], m >= 1 (m <= 1<<20)
+ *   cuts     device int32 [count][p-1], row-major, each row a valid cut vector
+ *   k        device int32 [count] in [1, AP_MAX_K], or NULL for k = 1
+ *   count    >= 0
+ *   time_ns  device int64 [count] (written)
+ *   master   device int32 [count] (written) or NULL to skip the critical path
+ * Asynchronous on `stream`.  INVALID cut vectors or k produce time_ns = -1 and
+ * master = -1 for that row (validated on the device, the call still returns OK).
+ * RANGE if the overflow guard m*(sum f + sum b) + 2m(p-1)*max comm >= 2^62 trips.
+ */
+ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                        const int32_t* k, int64_t count, int64_t* time_ns, int32_t* master,
+                        ap_stream_t stream);
+
+/*
+ * ap_search_exhaustive -- exact argmin over a contiguous slice of the search space.
+ * Simulates every partition with lex rank in [rank_lo, rank_hi) for every
+ * k in [k_lo, k_hi] (each (partition, k) pair fully simulated, no pruning) and
+ * writes ONE packed int64 key to device memory:
+ *     key = T << rb | (rank*(k_hi-k_lo+1) + k - k_lo),  rb = bitlen(N*K - 1),
+ * N = C(n-1,p-1), K = k_hi-k_lo+1, or INT64_MAX if the slice holds no candidate
+ * with T < T_ref+1, where T_ref = T(Algorithm 1 partition, k_lo)
+ * is an attained upper bound on the optimum.  The minimum key over all slices is
+ * the lexicographic min of (T, rank, k) ("Return the partition scheme
+ * with minimum iteration time"; reading Q15), so the keys of disjoint slices on
+ * different GPUs combine with one all_reduce(MIN) (BASELINE north_star).
+ *   key     device int64[1] (written)
+ * Synchronises `stream` once (to read T_ref), then launches asynchronously.
+ * Errors: INVALID (p, m, k range, empty or out-of-range rank slice), RANGE (overflow
+ * guard, or T_ref << rb does not fit in 63 bits), CUDA, NOMEM.
+ */
+ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                               int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
+                               int64_t* key, ap_stream_t stream);
+
+/*
+ * ap_search_heuristic -- AutoPipe's boundary-shifting heuristic (PAPER.md:147-198,
+ * steps 1, 3, 4; step 2 / Eq. (1) is adjust_mode 1, not yet supported), run as
+ * independent deterministic restarts r in [r_lo, r_hi), one GPU lane each.
+ * Restart 0 starts at the Algorithm 1 partition; restart r >= 1 at
+ * the seeded perturbation of DESIGN.md reading Q21 (splitmix64(seed ^ r<<32 ^ x),
+ * offsets in [-radius, radius]).  Each restart walks: if the master stage i is 0,
+ * stop; else simulate the children "move the first block of stage i to i-1"
+ * (+/- Algorithm 1 on the first i-1 stages) and "move the last block of stage i to
+ * i+1" (+/- Algorithm 1 on the first i stages); move to the
+ * child with master <= i and least (T, child order); stop if none.  A restart's
+ * result is the first-visited partition of least T among all it simulated.  k = 1.
+ *   key   device int64[1]: min over restarts of (T << 20 | r), INT64_MAX if none.
+ *   0 <= r_lo < r_hi <= 2^20, 0 <= radius <= 1<<20, adjust_mode must be 0.
+ * Synchronises `stream` once (overflow guard), then launches asynchronously.
+ */
+ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
+                              int32_t radius, uint32_t r_lo, uint32_t r_hi,
+                              int32_t adjust_mode, int64_t* key, ap_stream_t stream);
+
+typedef struct {
+  int64_t time_ns;          /* T of the decoded candidate                     */
+  uint64_t rank;            /* lex rank (mode 0) / rank of the cut vector (1) */
+  uint32_t restart;         /* winning restart (mode 1), 0 for mode 0         */
+  int32_t k;                /* slice pieces of micro-batch 0                  */
+  int32_t master;           /* master stage of the decoded candidate          */
+  int32_t p;                /* stages                                         */
+  int32_t cuts[AP_MAX_P - 1];
+} ap_result;
+
+/*
+ * ap_decode -- turn a reduced key into a plan (blocking).
+ *   mode 0: key from ap_search_exhaustive(k_lo, k_hi): unrank on the device and
+ *           re-simulate (T must equal the key's T; master from the critical path).
+ *   mode 1: key from ap_search_heuristic(seed, radius, adjust_mode): replay the
+ *           winning restart on the device to recover its cut vector.
+ * INVALID if key == INT64_MAX (empty search) or is not decodable.
+ */
+ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int32_t k_lo,
+                    int32_t k_hi, uint64_t seed, int32_t radius, int32_t adjust_mode,
+                    int64_t key, ap_result* out);
+
+/*
+ * ap_slice_sweep -- the Slicer's choice for one partition (§III-C;
+ * BASELINE north_star "micro-batch 0 sliced into k pieces"): T(k) for k = 1..k_max,
+ * best_k = argmin (T, k) (smallest k on ties).  Blocking.
+ *   cuts     host int32[p-1];  time_ns host int64[k_max] (written)
+ *   k_max in [1, AP_MAX_K]
+ */
+ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                         int32_t k_max, int64_t* time_ns, int32_t* best_k);
+
+typedef struct {
+  int32_t stage;       /* x                                        */
+  int32_t kind;        /* 0 = forward (FP), 1 = backward (BP)      */
+  int32_t microbatch;  /* micro-batch index j                      */
+  int32_t piece;       /* slice piece q of micro-batch 0's FP, else 0 */
+  int64_t start_ns;    /* compute start (after the receive Comm)   */
+  int64_t end_ns;      /* compute end                              */
+} ap_op;
+
+/*
+ * ap_critical_path -- the unique critical path (Fig. 4: the longest
+ * path of the AOE network, "closest to the last pipeline stage in the 1F1B phase";
+ * reading Q10) from F(0, mb 0, piece 0) to B(0, m-1), its master stage and T.
+ * Blocking.  cuts host int32[p-1]; ops host ap_op[cap] written source -> sink;
+ * *len = path length (also on CAPACITY, so the caller can retry).
+ */
+ap_status ap_critical_path(const ap_plan* plan, int32_t p, int32_t m, int32_t k,
+                           const int32_t* cuts, ap_op* ops, int32_t cap, int32_t* len,
+                           int32_t* master, int64_t* time_ns);
+
+/*
+ * ap_alg1 -- Algorithm 1: the min-max balanced partition of the
+ * n sub-layers into p stages by f+b (Comm unused, reading Q16; ties -> smallest
+ * split point).  Runs on the device; blocking.  cuts host int32[p-1]; value =
+ * the max stage load of that partition.
+ */
+ap_status ap_alg1(const ap_plan* plan, int32_t p, int32_t* cuts, int64_t* value);
+
+/* Details of the last ap_search_exhaustive launch on this thread (for benches):
+ * which sweep variant ran and its grid. */
+typedef struct {
+  int32_t fast_u32;        /* 1: exact u32 saturating sweep, 0: int64 sweep        */
+  int32_t exact_p;         /* 1: kernel specialised for this p, 0: generic        */
+  int32_t blocks, threads; /* grid                                                */
+  uint64_t chunk;          /* ranks per thread                                    */
+  int64_t t_ref;           /* T(Algorithm 1 partition, k_lo)                      */
+  int32_t rank_bits;       /* rb                                                  */
+  int32_t launches;        /* kernels launched by the call                        */
+} ap_launch_info;
+void ap_last_launch(ap_launch_info* info);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* AP_H_ */

@@ -1,0 +1,595 @@
+// ap_host.cu -- C-ABI implementation of include/ap.h.
+//
+// Host side only validates, allocates, launches and copies.  Every step of the
+// method (prefix sums, Algorithm 1, simulation, critical path, search, unranking,
+// restarts) runs in the kernels of ap_kernels.cu.  There is no CPU fallback: with
+// no sm_100 device every call fails with AP_ERR_CUDA.
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/ap.h"
+#include "ap_launch.h"
+
+namespace {
+
+thread_local std::string g_err;
+thread_local ap_launch_info g_last{};
+
+ap_status fail(ap_status st, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return st;
+}
+
+#define AP_CUDA(expr)                                                                 \
+  do {                                                                                \
+    cudaError_t e__ = (expr);                                                         \
+    if (e__ != cudaSuccess)                                                           \
+      return fail(e__ == cudaErrorMemoryAllocation ? AP_ERR_NOMEM : AP_ERR_CUDA,      \
+                  "%s: %s (%s:%d)", #expr, cudaGetErrorString(e__), __FILE__, __LINE__); \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+// Per-call device scratch, released stream-ordered.
+struct Scratch {
+  cudaStream_t s;
+  std::vector<void*> ptrs;
+  explicit Scratch(cudaStream_t st) : s(st) {}
+  cudaError_t get(void** p, size_t bytes) {
+    cudaError_t e = cudaMallocAsync(p, bytes < 16 ? 16 : bytes, s);
+    if (e == cudaSuccess) ptrs.push_back(*p);
+    return e;
+  }
+  ~Scratch() {
+    for (void* p : ptrs) cudaFreeAsync(p, s);
+  }
+};
+
+int bitlen(unsigned __int128 v) {
+  int b = 0;
+  while (v) {
+    ++b;
+    v >>= 1;
+  }
+  return b;
+}
+
+uint64_t binom_sat(int a, int b) {
+  if (b < 0 || b > a) return 0;
+  unsigned __int128 r = 1;
+  for (int i = 1; i <= b; ++i) {
+    r = r * (unsigned)(a - b + i) / (unsigned)i;
+    if (r > (unsigned __int128)UINT64_MAX) return UINT64_MAX;
+  }
+  return (uint64_t)r;
+}
+
+}  // namespace
+
+struct ap_plan {
+  int n = 0, npad = 0, device = 0;
+  std::vector<int64_t> f, b, act, comm;
+  int64_t sum_f = 0, sum_b = 0, max_comm = 0;
+  uint64_t link = 0;
+  int64_t* d_tab = nullptr;
+  uint64_t* d_binom = nullptr;
+  apk::DevTables dev() const { return apk::DevTables{d_tab, d_binom, n, npad}; }
+};
+
+extern "C" {
+
+const char* ap_last_error(void) { return g_err.c_str(); }
+
+const char* ap_version(void) { return "autopipe-b200 0.1 (sm_100a)"; }
+
+void ap_last_launch(ap_launch_info* info) {
+  if (info) *info = g_last;
+}
+
+ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns,
+                         const int64_t* act_bytes, uint64_t link_bytes_per_s, int32_t device,
+                         ap_plan** out) {
+  g_err.clear();
+  if (!out) return fail(AP_ERR_INVALID, "out is NULL");
+  *out = nullptr;
+  if (n < 1 || n > AP_MAX_N) return fail(AP_ERR_INVALID, "n=%d outside [1, %d]", n, AP_MAX_N);
+  if (!fwd_ns || !bwd_ns || !act_bytes) return fail(AP_ERR_INVALID, "NULL table");
+  if (link_bytes_per_s == 0) return fail(AP_ERR_INVALID, "link_bytes_per_s = 0");
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
+    return fail(AP_ERR_CUDA, "no CUDA device (the library has no CPU fallback)");
+  if (device < 0 || device >= ndev) return fail(AP_ERR_INVALID, "device %d of %d", device, ndev);
+  cudaDeviceProp prop;
+  AP_CUDA(cudaGetDeviceProperties(&prop, device));
+  if (prop.major != 10)
+    return fail(AP_ERR_CUDA, "device %d is sm_%d%d; this library is built for sm_100a", device,
+                prop.major, prop.minor);
+  ap_plan* P = new ap_plan();
+  P->n = n;
+  P->npad = (n + 1) & ~1;  // even => 16-byte multiple per array (TMA bulk copy)
+  P->device = device;
+  P->link = link_bytes_per_s;
+  P->f.assign(fwd_ns, fwd_ns + n);
+  P->b.assign(bwd_ns, bwd_ns + n);
+  P->act.assign(act_bytes, act_bytes + n);
+  P->comm.assign(n, 0);
+  unsigned __int128 sf = 0, sb = 0;
+  for (int i = 0; i < n; ++i) {
+    if (fwd_ns[i] < 0 || bwd_ns[i] < 0 || act_bytes[i] < 0) {
+      delete P;
+      return fail(AP_ERR_INVALID, "negative entry at sub-layer %d", i);
+    }
+    sf += (uint64_t)fwd_ns[i];
+    sb += (uint64_t)bwd_ns[i];
+    // Comm = ceil(bytes * 1e9 / bandwidth), exact in 128 bits (reading Q4, Q25)
+    const unsigned __int128 num = (unsigned __int128)(uint64_t)act_bytes[i] * 1000000000u;
+    const unsigned __int128 q = (num + link_bytes_per_s - 1) / link_bytes_per_s;
+    if (q >= ((unsigned __int128)1 << 62)) {
+      delete P;
+      return fail(AP_ERR_RANGE, "comm of sub-layer %d overflows", i);
+    }
+    if (i < n - 1) P->comm[i] = (int64_t)q;
+  }
+  if (sf >= ((unsigned __int128)1 << 62) || sb >= ((unsigned __int128)1 << 62)) {
+    delete P;
+    return fail(AP_ERR_RANGE, "sum of f or b >= 2^62");
+  }
+  P->sum_f = (int64_t)sf;
+  P->sum_b = (int64_t)sb;
+  for (int i = 0; i < n - 1; ++i) P->max_comm = P->comm[i] > P->max_comm ? P->comm[i] : P->max_comm;
+  std::vector<int64_t> tab(3 * (size_t)P->npad, 0);
+  for (int i = 0; i < n; ++i) {
+    tab[i] = P->f[i];
+    tab[P->npad + i] = P->b[i];
+    tab[2 * P->npad + i] = P->comm[i];
+  }
+  std::vector<uint64_t> binom((size_t)(n + 1) * 33, 0);
+  for (int a = 0; a <= n; ++a)
+    for (int bb = 0; bb <= 32 && bb <= a; ++bb) binom[(size_t)a * 33 + bb] = binom_sat(a, bb);
+  DeviceGuard g(device);
+  cudaError_t e = cudaMalloc((void**)&P->d_tab, tab.size() * 8);
+  if (e == cudaSuccess) e = cudaMalloc((void**)&P->d_binom, binom.size() * 8);
+  if (e == cudaSuccess) e = cudaMemcpy(P->d_tab, tab.data(), tab.size() * 8, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess)
+    e = cudaMemcpy(P->d_binom, binom.data(), binom.size() * 8, cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) {
+    ap_plan_destroy(P);
+    return fail(e == cudaErrorMemoryAllocation ? AP_ERR_NOMEM : AP_ERR_CUDA, "plan upload: %s",
+                cudaGetErrorString(e));
+  }
+  *out = P;
+  return AP_OK;
+}
+
+void ap_plan_destroy(ap_plan* plan) {
+  if (!plan) return;
+  {
+    DeviceGuard g(plan->device);
+    if (plan->d_tab) cudaFree(plan->d_tab);
+    if (plan->d_binom) cudaFree(plan->d_binom);
+  }
+  delete plan;
+}
+
+ap_status ap_plan_info(const ap_plan* plan, int32_t* n, int64_t* comm_ns) {
+  if (!plan) return fail(AP_ERR_INVALID, "plan is NULL");
+  if (n) *n = plan->n;
+  if (comm_ns) memcpy(comm_ns, plan->comm.data(), plan->comm.size() * 8);
+  return AP_OK;
+}
+
+ap_status ap_count(int32_t n, int32_t p, uint64_t* out) {
+  if (!out) return fail(AP_ERR_INVALID, "out is NULL");
+  if (n < 1 || p < 1 || p > n) return fail(AP_ERR_INVALID, "need 1 <= p <= n (p=%d, n=%d)", p, n);
+  unsigned __int128 r = 1;
+  const int a = n - 1, bb = p - 1;
+  for (int i = 1; i <= bb; ++i) {
+    r = r * (unsigned)(a - bb + i) / (unsigned)i;
+    if (r >= ((unsigned __int128)1 << 63)) return fail(AP_ERR_RANGE, "C(%d,%d) >= 2^63", a, bb);
+  }
+  *out = (uint64_t)r;
+  return AP_OK;
+}
+
+}  // extern "C"
+
+namespace {
+
+ap_status check_pm(const ap_plan* plan, int p, int m) {
+  if (!plan) return fail(AP_ERR_INVALID, "plan is NULL");
+  if (p < 1 || p > plan->n || p > AP_MAX_P)
+    return fail(AP_ERR_INVALID, "p=%d outside [1, min(n=%d, %d)]", p, plan->n, AP_MAX_P);
+  if (m < 1 || m > (1 << 20)) return fail(AP_ERR_INVALID, "m=%d outside [1, 2^20]", m);
+  // overflow guard: every finish time is at most the sum of all op weights
+  const unsigned __int128 tot = (unsigned __int128)m * (uint64_t)(plan->sum_f + plan->sum_b) +
+                                (unsigned __int128)2 * m * (p - 1) * (uint64_t)plan->max_comm;
+  if (tot >= ((unsigned __int128)1 << 62)) return fail(AP_ERR_RANGE, "overflow guard: total >= 2^62");
+  return AP_OK;
+}
+
+cudaStream_t S_(ap_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
+
+}  // namespace
+
+extern "C" {
+
+ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                        const int32_t* k, int64_t count, int64_t* time_ns, int32_t* master,
+                        ap_stream_t stream) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (count < 0) return fail(AP_ERR_INVALID, "count < 0");
+  if (count == 0) return AP_OK;
+  if (!time_ns || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL output/cuts");
+  DeviceGuard g(plan->device);
+  int launches = 0;
+  static const int32_t kDummy = 0;
+  (void)kDummy;
+  AP_CUDA(apk::launch_eval(plan->dev(), p, m, p > 1 ? cuts : nullptr, p - 1, k, 1, 0, count,
+                           time_ns, master, S_(stream), &launches));
+  return AP_OK;
+}
+
+}  // extern "C"
+
+namespace {
+
+// Algorithm 1 on the device into scratch; returns device pointers.
+ap_status run_alg1(const ap_plan* plan, int p, Scratch& sc, int16_t** d_arg, int32_t** d_cuts,
+                   int64_t** d_val) {
+  AP_CUDA(sc.get((void**)d_arg, (size_t)(plan->n + 1) * (p + 1) * 2));
+  AP_CUDA(sc.get((void**)d_cuts, 4 * 32));
+  AP_CUDA(sc.get((void**)d_val, 8));
+  AP_CUDA(apk::launch_alg1(plan->dev(), p, *d_arg, *d_cuts, *d_val, sc.s));
+  return AP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+ap_status ap_alg1(const ap_plan* plan, int32_t p, int32_t* cuts, int64_t* value) {
+  g_err.clear();
+  if (!plan) return fail(AP_ERR_INVALID, "plan is NULL");
+  if (p < 1 || p > plan->n || p > AP_MAX_P) return fail(AP_ERR_INVALID, "p=%d", p);
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  ap_status st;
+  {
+    Scratch sc(s);
+    int16_t* arg;
+    int32_t* dc;
+    int64_t* dv;
+    st = run_alg1(plan, p, sc, &arg, &dc, &dv);
+    if (st == AP_OK) {
+      int64_t v = 0;
+      std::vector<int32_t> hc(32, 0);
+      cudaError_t e = cudaMemcpyAsync(hc.data(), dc, 4 * 32, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&v, dv, 8, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess) st = fail(AP_ERR_CUDA, "alg1: %s", cudaGetErrorString(e));
+      else {
+        if (cuts && p > 1) memcpy(cuts, hc.data(), 4 * (p - 1));
+        if (value) *value = v;
+      }
+    }
+  }
+  cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  return st;
+}
+
+ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                               int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int64_t* key,
+                               ap_stream_t stream) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (!key) return fail(AP_ERR_INVALID, "key is NULL");
+  if (k_lo < 1 || k_hi < k_lo || k_hi > AP_MAX_K)
+    return fail(AP_ERR_INVALID, "k range [%d, %d] outside [1, %d]", k_lo, k_hi, AP_MAX_K);
+  uint64_t N;
+  st = ap_count(plan->n, p, &N);
+  if (st != AP_OK) return st;
+  if (rank_lo >= rank_hi || rank_hi > N)
+    return fail(AP_ERR_INVALID, "rank slice [%llu, %llu) empty or beyond N=%llu",
+                (unsigned long long)rank_lo, (unsigned long long)rank_hi, (unsigned long long)N);
+  const unsigned __int128 NK = (unsigned __int128)N * (unsigned)(k_hi - k_lo + 1);
+  const int rb = bitlen(NK - 1);
+  cudaStream_t s = S_(stream);
+  DeviceGuard g(plan->device);
+  ap_launch_info info{};
+  Scratch sc(s);
+  int16_t* d_arg;
+  int32_t* d_a1;
+  int64_t* d_val;
+  st = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
+  if (st != AP_OK) return st;
+  int64_t* d_tref;
+  AP_CUDA(sc.get((void**)&d_tref, 8));
+  int launches = 1;
+  AP_CUDA(apk::launch_eval(plan->dev(), p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 0, 1,
+                           d_tref, nullptr, s, &launches));
+  int64_t tref = 0;
+  AP_CUDA(cudaMemcpyAsync(&tref, d_tref, 8, cudaMemcpyDeviceToHost, s));
+  AP_CUDA(cudaStreamSynchronize(s));
+  if (tref < 0) return fail(AP_ERR_CUDA, "T_ref evaluation failed");
+  if (rb >= 63 || (uint64_t)tref >= ((1ull << (63 - rb)) - 1))
+    return fail(AP_ERR_RANGE, "key packing: T_ref=%lld needs %d bits + %d rank bits > 63",
+                (long long)tref, bitlen((unsigned __int128)tref), rb);
+  // exact u32 saturating fast path: S = T_ref + 1, rows between
+  // clamps <= max(p, 4) + 2, each row adds at most W_row to any running value.
+  const uint64_t S = (uint64_t)tref + 1;
+  const unsigned __int128 wrow = (unsigned __int128)(plan->sum_f + plan->sum_b) +
+                                 (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm;
+  const int seg = (p > 4 ? p : 4) + 2;
+  int want_u32 = ((unsigned __int128)S + wrow * seg) < ((unsigned __int128)1 << 32);
+  // test/bench overrides: AP_SWEEP=int64 disables the u32 path, AP_SWEEP=generic
+  // also the p-specialised kernel (both remain exact)
+  const char* ov = getenv("AP_SWEEP");
+  int force_generic = 0;
+  if (ov && strcmp(ov, "int64") == 0) want_u32 = 0;
+  if (ov && strcmp(ov, "generic") == 0) { want_u32 = 0; force_generic = 1; }
+  apk::SweepPlan sp{};
+  AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, S, rb, want_u32,
+                            force_generic, reinterpret_cast<unsigned long long*>(key), s, &sp));
+  launches += 2;
+  info.fast_u32 = sp.fast_u32;
+  info.exact_p = sp.exact_p;
+  info.blocks = sp.blocks;
+  info.threads = sp.threads;
+  info.chunk = sp.chunk;
+  info.t_ref = tref;
+  info.rank_bits = rb;
+  info.launches = launches;
+  g_last = info;
+  return AP_OK;
+}
+
+ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
+                              int32_t radius, uint32_t r_lo, uint32_t r_hi, int32_t adjust_mode,
+                              int64_t* key, ap_stream_t stream) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (!key) return fail(AP_ERR_INVALID, "key is NULL");
+  if (adjust_mode != 0) return fail(AP_ERR_INVALID, "adjust_mode %d not supported (only 0)", adjust_mode);
+  if (r_lo >= r_hi || r_hi > (1u << 20)) return fail(AP_ERR_INVALID, "restart range [%u, %u)", r_lo, r_hi);
+  if (radius < 0 || radius > (1 << 20)) return fail(AP_ERR_INVALID, "radius %d", radius);
+  cudaStream_t s = S_(stream);
+  DeviceGuard g(plan->device);
+  Scratch sc(s);
+  int16_t* d_arg;
+  int32_t* d_a1;
+  int64_t* d_val;
+  st = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
+  if (st != AP_OK) return st;
+  unsigned int* d_ctr;
+  AP_CUDA(sc.get((void**)&d_ctr, 16));
+  AP_CUDA(apk::launch_heuristic(plan->dev(), p, m, seed, radius, r_lo, r_hi, d_arg, d_a1, d_ctr,
+                                reinterpret_cast<unsigned long long*>(key), nullptr, s));
+  ap_launch_info info{};
+  info.launches = 3;
+  g_last = info;
+  return AP_OK;
+}
+
+ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int32_t k_lo,
+                    int32_t k_hi, uint64_t seed, int32_t radius, int32_t adjust_mode, int64_t key,
+                    ap_result* out) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (!out) return fail(AP_ERR_INVALID, "out is NULL");
+  if (key == INT64_MAX || key < 0) return fail(AP_ERR_INVALID, "empty key (no candidate found)");
+  memset(out, 0, sizeof *out);
+  out->p = p;
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  ap_status res = AP_OK;
+  {
+    Scratch sc(s);
+    int32_t* d_cuts = nullptr;
+    int32_t* d_master = nullptr;
+    int64_t* d_T = nullptr;
+    int64_t keyT = 0;
+    int kk = 1;
+    cudaError_t e = sc.get((void**)&d_cuts, 4 * 32);
+    if (e == cudaSuccess) e = sc.get((void**)&d_master, 16);
+    if (e == cudaSuccess) e = sc.get((void**)&d_T, 16);
+    if (e != cudaSuccess) res = fail(AP_ERR_NOMEM, "decode scratch");
+    if (res == AP_OK && mode == 0) {
+      uint64_t N;
+      res = ap_count(plan->n, p, &N);
+      if (res == AP_OK) {
+        if (k_lo < 1 || k_hi < k_lo || k_hi > AP_MAX_K) res = fail(AP_ERR_INVALID, "k range");
+      }
+      if (res == AP_OK) {
+        const uint64_t K = (uint64_t)(k_hi - k_lo + 1);
+        const int rb = bitlen((unsigned __int128)N * K - 1);
+        keyT = (int64_t)((uint64_t)key >> rb);
+        const uint64_t idx = (uint64_t)key & ((rb == 0) ? 0ull : ((1ull << rb) - 1));
+        const uint64_t rank = idx / K;
+        kk = k_lo + (int)(idx % K);
+        if (rank >= N) res = fail(AP_ERR_INVALID, "rank %llu >= N", (unsigned long long)rank);
+        out->rank = rank;
+        out->k = kk;
+        if (res == AP_OK && p > 1) {
+          e = apk::launch_unrank(plan->dev(), p, rank, d_cuts, s);
+          if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "unrank: %s", cudaGetErrorString(e));
+        }
+      }
+    } else if (res == AP_OK && mode == 1) {
+      if (adjust_mode != 0) res = fail(AP_ERR_INVALID, "adjust_mode %d", adjust_mode);
+      keyT = key >> 20;
+      const uint32_t r = (uint32_t)(key & ((1 << 20) - 1));
+      out->restart = r;
+      out->k = 1;
+      kk = 1;
+      int16_t* d_arg;
+      int32_t* d_a1;
+      int64_t* d_val;
+      unsigned int* d_ctr;
+      unsigned long long* d_key;
+      if (res == AP_OK) res = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
+      if (res == AP_OK) {
+        e = sc.get((void**)&d_ctr, 16);
+        if (e == cudaSuccess) e = sc.get((void**)&d_key, 16);
+        if (e == cudaSuccess)
+          e = apk::launch_heuristic(plan->dev(), p, m, seed, radius, r, r + 1, d_arg, d_a1, d_ctr,
+                                    d_key, d_cuts, s);
+        if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "replay: %s", cudaGetErrorString(e));
+      }
+    } else if (res == AP_OK) {
+      res = fail(AP_ERR_INVALID, "mode %d", mode);
+    }
+    if (res == AP_OK) {
+      int launches = 0;
+      e = apk::launch_eval(plan->dev(), p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, kk, 0, 1, d_T,
+                           d_master, s, &launches);
+      int32_t hc[32] = {0};
+      int64_t T = -1;
+      int32_t M = -1;
+      if (e == cudaSuccess) e = cudaMemcpyAsync(hc, d_cuts, 4 * 32, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&T, d_T, 8, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&M, d_master, 4, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess) {
+        res = fail(AP_ERR_CUDA, "decode eval: %s", cudaGetErrorString(e));
+      } else {
+        if (p > 1) memcpy(out->cuts, hc, 4 * (p - 1));
+        out->time_ns = T;
+        out->master = M;
+        if (T != keyT)
+          res = fail(AP_ERR_INVALID, "key does not decode: T(key)=%lld, re-simulated %lld",
+                     (long long)keyT, (long long)T);
+        if (mode == 1 && res == AP_OK) {
+          // rank of the heuristic winner, for reference (host arithmetic on the result)
+          uint64_t r = 0;
+          int prev = 0;
+          for (int x = 1; x <= p - 1; ++x) {
+            for (int v = prev + 1; v <= hc[x - 1] - 1; ++v) r += binom_sat(plan->n - 1 - v, p - 1 - x);
+            prev = hc[x - 1];
+          }
+          out->rank = r;
+        }
+      }
+    }
+  }
+  cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  return res;
+}
+
+ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                         int32_t k_max, int64_t* time_ns, int32_t* best_k) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (k_max < 1 || k_max > AP_MAX_K) return fail(AP_ERR_INVALID, "k_max=%d", k_max);
+  if (!time_ns || !best_k || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL argument");
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  ap_status res = AP_OK;
+  {
+    Scratch sc(s);
+    int32_t* d_cuts;
+    int64_t* d_T;
+    cudaError_t e = sc.get((void**)&d_cuts, 4 * 32);
+    if (e == cudaSuccess) e = sc.get((void**)&d_T, 8 * (size_t)k_max);
+    if (e == cudaSuccess && p > 1)
+      e = cudaMemcpyAsync(d_cuts, cuts, 4 * (size_t)(p - 1), cudaMemcpyHostToDevice, s);
+    int launches = 0;
+    if (e == cudaSuccess)
+      e = apk::launch_eval(plan->dev(), p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, 1, 1, k_max,
+                           d_T, nullptr, s, &launches);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(time_ns, d_T, 8 * (size_t)k_max, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "slice sweep: %s", cudaGetErrorString(e));
+  }
+  cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  if (res != AP_OK) return res;
+  if (time_ns[0] < 0) return fail(AP_ERR_INVALID, "invalid cut vector");
+  int bk = 1;
+  for (int q = 2; q <= k_max; ++q)
+    if (time_ns[q - 1] < time_ns[bk - 1]) bk = q;  // min (T, k)
+  *best_k = bk;
+  return AP_OK;
+}
+
+ap_status ap_critical_path(const ap_plan* plan, int32_t p, int32_t m, int32_t k,
+                           const int32_t* cuts, ap_op* ops, int32_t cap, int32_t* len,
+                           int32_t* master, int64_t* time_ns) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (k < 1 || k > AP_MAX_K) return fail(AP_ERR_INVALID, "k=%d", k);
+  if (cap < 0 || (cap > 0 && !ops) || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL argument");
+  static_assert(sizeof(ap_op) == sizeof(apk::OpRec), "ap_op layout");
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  ap_status res = AP_OK;
+  int32_t lm[2] = {-1, -1};
+  int64_t T = -1;
+  {
+    Scratch sc(s);
+    int32_t *d_cuts, *d_lm;
+    int64_t* d_T;
+    apk::OpRec* d_ops;
+    void* d_scr;
+    const int cap_dev = cap > 0 ? cap : 1;
+    cudaError_t e = sc.get((void**)&d_cuts, 4 * 32);
+    if (e == cudaSuccess) e = sc.get((void**)&d_lm, 16);
+    if (e == cudaSuccess) e = sc.get((void**)&d_T, 16);
+    if (e == cudaSuccess) e = sc.get((void**)&d_ops, sizeof(apk::OpRec) * (size_t)cap_dev);
+    if (e == cudaSuccess) e = sc.get(&d_scr, apk::cpath_scratch_bytes(p, m));
+    if (e == cudaSuccess && p > 1)
+      e = cudaMemcpyAsync(d_cuts, cuts, 4 * (size_t)(p - 1), cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess)
+      e = apk::launch_cpath(plan->dev(), p, m, k, d_cuts, d_ops, cap, d_lm, d_T, d_scr, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(lm, d_lm, 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&T, d_T, 8, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e == cudaSuccess && lm[0] > 0 && lm[0] <= cap)
+      e = cudaMemcpyAsync(ops, d_ops, sizeof(ap_op) * (size_t)lm[0], cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "critical path: %s", cudaGetErrorString(e));
+  }
+  cudaStreamSynchronize(s);
+  cudaStreamDestroy(s);
+  if (res != AP_OK) return res;
+  if (lm[0] < 0) return fail(AP_ERR_INVALID, "invalid cut vector");
+  if (len) *len = lm[0];
+  if (master) *master = lm[1];
+  if (time_ns) *time_ns = T;
+  if (lm[0] > cap) return fail(AP_ERR_CAPACITY, "path has %d ops, cap %d", lm[0], cap);
+  return AP_OK;
+}
+
+}  // extern "C"

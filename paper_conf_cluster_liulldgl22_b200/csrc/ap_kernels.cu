@@ -1,0 +1,1030 @@
+// ap_kernels.cu -- sm_100a kernels of the AutoPipe planner/slicer hot path.
+//
+//   k_sweep_exact<P,V>  K1 exhaustive sweep, p == P, m >= P.  V = uint32_t is the
+//                       exact saturating fast path, V = uint64_t
+//                       the plain int64 one.  Per thread: unrank once, lex
+//                       successor, row sweep per (rank, k), register argmin,
+//                       warp-shuffle -> block -> atomicMin (K5).
+//   k_sweep_generic<P>  K1 for any p <= P and any m (exact int64, runtime p).
+//   k_eval<P>           K2 thread-per-candidate T (+ master via bits/backtrack).
+//   k_heur<P>           K3 heuristic restarts, one lane per restart, refilled from
+//                       an atomic restart counter.
+//   k_alg1              Algorithm 1 DP, one CTA.
+//   k_cpath<P>          critical path with op times for one candidate.
+//   k_unrank, k_init    decode / key init.
+// Every kernel starts with the K4 prologue (TMA bulk copy of the tables into
+// shared memory + warp-shuffle prefix sums), see ap_device.cuh.
+#include <climits>
+#include <cstdio>
+
+#include "ap_device.cuh"
+#include "ap_launch.h"
+
+namespace apk {
+using namespace apdev;
+
+// ===========================================================================
+// K1 fast sweep.
+template <typename V>
+AP_DEV_INLINE V vmax(V a, V b) {
+  return a > b ? a : b;
+}
+template <typename V>
+AP_DEV_INLINE V vmin(V a, V b) {
+  return a < b ? a : b;
+}
+
+// floor(v / k) for the u32 path: one umulhi with M_k = floor(2^32/k) (k=1:
+// 2^32-1) under-estimates by at most 1, fixed by one compare.
+AP_DEV_INLINE uint32_t divk(uint32_t v, uint32_t k, uint32_t M) {
+  uint32_t q = __umulhi(v, M);
+  const uint32_t r = v - q * k;
+  return q + (r >= k ? 1u : 0u);
+}
+AP_DEV_INLINE uint64_t divk(uint64_t v, uint32_t k, uint32_t) { return v / k; }
+
+template <int P, typename V>
+AP_DEV_INLINE void clamp_state(V (&FF)[P], V (&L)[P], V S) {
+  if constexpr (sizeof(V) == 4) {
+#pragma unroll
+    for (int x = 0; x < P; ++x) {
+      FF[x] = vmin(FF[x], S);
+      L[x] = vmin(L[x], S);
+    }
+  }
+}
+
+// One steady 1F1B row (rows r = P..m-1): every stage does F then B.
+template <int P, typename V>
+AP_DEV_INLINE void row_steady(V (&FF)[P], V (&L)[P], const V (&wF)[P], const V (&wB)[P]) {
+#pragma unroll
+  for (int x = P - 1; x >= 1; --x) FF[x] = vmax(FF[x - 1], L[x]) + wF[x];
+  FF[0] = L[0] + wF[0];
+  V b = FF[P - 1] + wB[P - 1];
+  L[P - 1] = b;
+#pragma unroll
+  for (int x = P - 2; x >= 0; --x) {
+    b = vmax(b, FF[x]) + wB[x];
+    L[x] = b;
+  }
+}
+
+// Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
+template <int P, typename V>
+AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const V (&Fr)[P],
+                         const V (&Ci)[P], uint32_t Mk, V S) {
+  V FF[P], L[P];
+  // micro-batch 0's forward, sliced into k pieces (reading Q6)
+  if (k == 1) {
+    FF[0] = wF[0];
+#pragma unroll
+    for (int x = 1; x < P; ++x) FF[x] = FF[x - 1] + wF[x];
+  } else {
+    V a[P], al[P];
+#pragma unroll
+    for (int x = 0; x < P; ++x) {
+      a[x] = divk(Fr[x], (uint32_t)k, Mk) + ((x > 0) ? divk(Ci[x], (uint32_t)k, Mk) : V(0));
+      al[x] = wF[x] - V(k - 1) * a[x];
+      FF[x] = 0;
+    }
+    for (int q = 0; q < k - 1; ++q) {
+      FF[0] = FF[0] + a[0];
+#pragma unroll
+      for (int x = 1; x < P; ++x) FF[x] = vmax(FF[x - 1], FF[x]) + a[x];
+    }
+    FF[0] = FF[0] + al[0];
+#pragma unroll
+    for (int x = 1; x < P; ++x) FF[x] = vmax(FF[x - 1], FF[x]) + al[x];
+  }
+  // warm-up rows r = 1..P-2: stage x <= r-1 does F(x, r-x); L == FF here
+#pragma unroll
+  for (int r = 1; r <= P - 2; ++r) {
+#pragma unroll
+    for (int x = r - 1; x >= 1; --x) FF[x] = vmax(FF[x - 1], FF[x]) + wF[x];
+    FF[0] = FF[0] + wF[0];
+  }
+#pragma unroll
+  for (int x = 0; x < P; ++x) L[x] = FF[x];
+  // row P-1: stages 0..P-2 do F(x, P-1-x); F(P-1, 0) was a piece; all do B(x, 0)
+  {
+#pragma unroll
+    for (int x = P - 2; x >= 1; --x) FF[x] = vmax(FF[x - 1], L[x]) + wF[x];
+    if (P >= 2) FF[0] = L[0] + wF[0];
+    V b = FF[P - 1] + wB[P - 1];
+    L[P - 1] = b;
+#pragma unroll
+    for (int x = P - 2; x >= 0; --x) {
+      b = vmax(b, FF[x]) + wB[x];
+      L[x] = b;
+    }
+  }
+  clamp_state<P, V>(FF, L, S);
+  // steady rows r = P..m-1
+  constexpr int U = (P <= 8) ? 4 : 2;
+  int rem = m - P;
+  for (; rem >= U; rem -= U) {
+#pragma unroll
+    for (int u = 0; u < U; ++u) row_steady<P, V>(FF, L, wF, wB);
+    clamp_state<P, V>(FF, L, S);
+  }
+  for (; rem > 0; --rem) row_steady<P, V>(FF, L, wF, wB);
+  clamp_state<P, V>(FF, L, S);
+  // cool-down rows r = m+c, c = 0..P-2: F only on stages x >= c+1
+#pragma unroll
+  for (int c = 0; c <= P - 2; ++c) {
+#pragma unroll
+    for (int x = P - 1; x >= c + 1; --x) FF[x] = vmax(FF[x - 1], L[x]) + wF[x];
+    V b = FF[P - 1] + wB[P - 1];
+    L[P - 1] = b;
+#pragma unroll
+    for (int x = P - 2; x >= 0; --x) {
+      const V in = (x >= c + 1) ? FF[x] : L[x];
+      b = vmax(b, in) + wB[x];
+      L[x] = b;
+    }
+  }
+  return L[0];
+}
+
+struct SweepArgs {
+  DevTables t;
+  int p, m, k_lo, k_hi;
+  uint64_t rank_lo, rank_hi, chunk;
+  uint64_t S;
+  int rb;
+  unsigned long long* key;
+};
+
+AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
+  return (a < 0 || b < 0 || b > a) ? 0ull : binom[a * 33 + b];
+}
+
+// Block-level min of a u64 key, one atomicMin per CTA.
+AP_DEV_INLINE void block_min_atomic(unsigned long long v, unsigned long long* out) {
+  __shared__ unsigned long long s_warp[32];
+#pragma unroll
+  for (int o = 16; o >= 1; o >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, o));
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) s_warp[warp] = v;
+  __syncthreads();
+  if (warp == 0) {
+    const int nw = (blockDim.x + 31) >> 5;
+    v = (lane < nw) ? s_warp[lane] : 0x7fffffffffffffffull;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, o));
+    if (lane == 0 && v != 0x7fffffffffffffffull) atomicMin(out, v);
+  }
+}
+
+template <int P, typename V>
+__global__ void __launch_bounds__(256) k_sweep_exact(SweepArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int n = A.t.n;
+  // V-typed copies of the prefix sums / comm (u32 path: exact by the host's bound)
+  V* sPf = reinterpret_cast<V*>(smem + used);
+  V* sPb = sPf + (n + 1);
+  V* sC = sPb + (n + 1);
+  for (int i = threadIdx.x; i <= n; i += blockDim.x) {
+    sPf[i] = (V)T.Pf[i];
+    sPb[i] = (V)T.Pb[i];
+    if (i < n) sC[i] = (V)T.comm[i];
+  }
+  __syncthreads();
+
+  const int m = A.m, k_lo = A.k_lo, k_hi = A.k_hi;
+  const uint64_t K = (uint64_t)(k_hi - k_lo + 1);
+  const V S = (V)A.S;
+  V bestT = S;
+  uint64_t bestIdx = 0;
+  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t r0 = A.rank_lo + tid * A.chunk;
+  if (r0 < A.rank_hi) {
+    const uint64_t r1 = min(r0 + A.chunk, A.rank_hi);
+    // unrank r0 (reading O7 lex order)
+    int c[P + 1];
+    c[0] = 0;
+    c[P] = n;
+    {
+      uint64_t rr = r0;
+      int prev = 0;
+#pragma unroll
+      for (int x = 1; x <= P - 1; ++x) {
+        int v = prev + 1;
+        for (;;) {
+          const uint64_t cnt = binom_at(A.t.binom, n - 1 - v, P - 1 - x);
+          if (rr >= cnt) {
+            rr -= cnt;
+            ++v;
+          } else {
+            break;
+          }
+        }
+        c[x] = v;
+        prev = v;
+      }
+    }
+    for (uint64_t r = r0; r < r1; ++r) {
+      // stage weights (a3): compute + receiver-side comm
+      V wF[P], wB[P], Fr[P], Ci[P];
+#pragma unroll
+      for (int x = 0; x < P; ++x) {
+        const V Fx = sPf[c[x + 1]] - sPf[c[x]];
+        const V Bx = sPb[c[x + 1]] - sPb[c[x]];
+        const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
+        const V Cout = (x < P - 1) ? sC[c[x + 1] - 1] : V(0);
+        wF[x] = Fx + Cin;
+        wB[x] = Bx + Cout;
+        Fr[x] = Fx;
+        Ci[x] = Cin;
+      }
+      const uint64_t base = r * K;
+      for (int k = k_lo; k <= k_hi; ++k) {
+        const uint32_t Mk = (k == 1) ? 0xffffffffu : (uint32_t)((1ull << 32) / (uint32_t)k);
+        const V Tc = sim_fast<P, V>(m, k, wF, wB, Fr, Ci, Mk, S);
+        if (Tc < bestT) {
+          bestT = Tc;
+          bestIdx = base + (uint64_t)(k - k_lo);
+        }
+      }
+      // lexicographic successor (a2)
+      int pos = 0;
+#pragma unroll
+      for (int x = P - 1; x >= 1; --x)
+        if (pos == 0 && c[x] < n - (P - x)) pos = x;
+#pragma unroll
+      for (int x = 1; x <= P - 1; ++x) {
+        if (x == pos) c[x] = c[x] + 1;
+        else if (x > pos && pos > 0) c[x] = c[x - 1] + 1;
+      }
+    }
+  }
+  const unsigned long long key = (bestT < S)
+                                     ? (((unsigned long long)bestT << A.rb) | bestIdx)
+                                     : 0x7fffffffffffffffull;
+  block_min_atomic(key, A.key);
+}
+
+// Generic exhaustive sweep: runtime p <= P, any m, exact int64.
+template <int P>
+__global__ void __launch_bounds__(128) k_sweep_generic(SweepArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int n = A.t.n, p = A.p, m = A.m;
+  const uint64_t K = (uint64_t)(A.k_hi - A.k_lo + 1);
+  int64_t bestT = (int64_t)A.S;
+  uint64_t bestIdx = 0;
+  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t r0 = A.rank_lo + tid * A.chunk;
+  if (r0 < A.rank_hi) {
+    const uint64_t r1 = min(r0 + A.chunk, A.rank_hi);
+    int c[P + 1];
+#pragma unroll
+    for (int x = 0; x <= P; ++x) c[x] = n;
+    c[0] = 0;
+    {
+      uint64_t rr = r0;
+      int prev = 0;
+#pragma unroll
+      for (int x = 1; x <= P - 1; ++x) {
+        if (x <= p - 1) {
+          int v = prev + 1;
+          for (;;) {
+            const uint64_t cnt = binom_at(A.t.binom, n - 1 - v, p - 1 - x);
+            if (rr >= cnt) {
+              rr -= cnt;
+              ++v;
+            } else {
+              break;
+            }
+          }
+          c[x] = v;
+          prev = v;
+        }
+      }
+    }
+    BitsRef nob{nullptr, 0};
+    TimesRef not_{nullptr, nullptr, nullptr};
+    uint32_t pb[P];
+    for (uint64_t r = r0; r < r1; ++r) {
+      int64_t F[P], B[P], C[P];
+      stage_costs<P>(T, p, c, F, B, C);
+      for (int k = A.k_lo; k <= A.k_hi; ++k) {
+        const int64_t Tc = sim_exact<P, 0>(p, m, k, F, B, C, nob, pb, not_);
+        if (Tc < bestT) {
+          bestT = Tc;
+          bestIdx = r * K + (uint64_t)(k - A.k_lo);
+        }
+      }
+      int pos = 0;
+#pragma unroll
+      for (int x = P - 1; x >= 1; --x)
+        if (x <= p - 1 && pos == 0 && c[x] < n - (p - x)) pos = x;
+#pragma unroll
+      for (int x = 1; x <= P - 1; ++x) {
+        if (x <= p - 1) {
+          if (x == pos) c[x] = c[x] + 1;
+          else if (x > pos && pos > 0) c[x] = c[x - 1] + 1;
+        }
+      }
+    }
+  }
+  const unsigned long long key = (bestT < (int64_t)A.S)
+                                     ? (((unsigned long long)bestT << A.rb) | bestIdx)
+                                     : 0x7fffffffffffffffull;
+  block_min_atomic(key, A.key);
+}
+
+__global__ void k_init_key(unsigned long long* key) { *key = 0x7fffffffffffffffull; }
+
+// ===========================================================================
+// K2 eval.
+struct EvalArgs {
+  DevTables t;
+  int p, m;
+  const int32_t* cuts;
+  int cuts_stride;
+  const int32_t* kptr;
+  int k_const, k_iota;
+  int64_t count;
+  int64_t* time_ns;
+  int32_t* master;
+  uint32_t* gbits;  // global bit scratch when shared memory is too small (or null)
+};
+
+template <int P>
+AP_DEV_INLINE bool load_cuts(const int32_t* row, int p, int n, int (&c)[P + 1]) {
+  bool ok = true;
+#pragma unroll
+  for (int x = 0; x <= P; ++x) c[x] = n;
+  c[0] = 0;
+  int prev = 0;
+#pragma unroll
+  for (int x = 1; x <= P - 1; ++x) {
+    if (x <= p - 1) {
+      const int v = row[x - 1];
+      ok = ok && (v > prev) && (v <= n - 1);
+      c[x] = v;
+      prev = v;
+    }
+  }
+  return ok;
+}
+
+template <int P>
+__global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= A.count) return;
+  const int p = A.p, m = A.m, n = A.t.n;
+  int c[P + 1];
+  const bool okc = load_cuts<P>(A.cuts + (size_t)i * A.cuts_stride, p, n, c);
+  const int k = A.kptr ? A.kptr[i] : (A.k_iota ? (int)(i + 1) : A.k_const);
+  if (!okc || k < 1 || k > kMaxK) {
+    A.time_ns[i] = -1;
+    if (A.master) A.master[i] = -1;
+    return;
+  }
+  int64_t F[P], B[P], C[P];
+  stage_costs<P>(T, p, c, F, B, C);
+  uint32_t pb[P];
+  TimesRef not_{nullptr, nullptr, nullptr};
+  if (A.master == nullptr) {
+    BitsRef nob{nullptr, 0};
+    A.time_ns[i] = sim_exact<P, 0>(p, m, k, F, B, C, nob, pb, not_);
+    return;
+  }
+  BitsRef br;
+  if (A.gbits) {
+    br.base = A.gbits + i;
+    br.stride = (int)A.count;
+  } else {
+    uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + ((used + 15) & ~size_t(15)));
+    br.base = sbits + threadIdx.x;
+    br.stride = blockDim.x;
+  }
+  A.time_ns[i] = sim_exact<P, 1>(p, m, k, F, B, C, br, pb, not_);
+  int len;
+  A.master[i] = backtrack_master<P>(p, m, k, br, pb, &len, NoEmit{});
+}
+
+// ===========================================================================
+// Algorithm 1, one CTA.  time[0][0] = 0, others +inf;
+// time[i][j] = min_k max(time[k][j-1], P[i]-P[k]) over k ascending, strict '<'
+// (smallest k wins ties); the arg table drives line 15's reconstruction.
+__global__ void __launch_bounds__(256) k_alg1(DevTables t, int p, int16_t* arg, int32_t* cuts,
+                                              int64_t* value) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
+  const int n = t.n, P1 = p + 1;
+  int64_t* tt = reinterpret_cast<int64_t*>(smem + ((used + 15) & ~size_t(15)));
+  // prefix_sum of f+b (line 6): Pf + Pb
+  for (int e = threadIdx.x; e < (n + 1) * P1; e += blockDim.x) {
+    tt[e] = (e == 0) ? 0 : INT64_MAX;
+    arg[e] = -1;
+  }
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int i = 1; i <= n; ++i) {
+    const int64_t Pi = T.Pf[i] + T.Pb[i];
+    const int jmax = min(p, i);
+    for (int j = 1 + warp; j <= jmax; j += nw) {
+      int64_t bv = INT64_MAX;
+      int bk = INT32_MAX;
+      for (int kk = lane; kk <= i - 1; kk += 32) {
+        const int64_t prev = tt[kk * P1 + (j - 1)];
+        const int64_t seg = Pi - (T.Pf[kk] + T.Pb[kk]);
+        const int64_t v = prev > seg ? prev : seg;
+        if (v < bv) {  // kk ascending within the lane: first wins
+          bv = v;
+          bk = kk;
+        }
+      }
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) {
+        const int64_t ov = __shfl_xor_sync(0xffffffffu, bv, o);
+        const int ok = __shfl_xor_sync(0xffffffffu, bk, o);
+        if (ov < bv || (ov == bv && ok < bk)) {
+          bv = ov;
+          bk = ok;
+        }
+      }
+      if (lane == 0 && bv != INT64_MAX) {
+        tt[i * P1 + j] = bv;
+        arg[i * P1 + j] = (int16_t)bk;
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    *value = tt[n * P1 + p];
+    int e = n;
+    for (int jj = p; jj >= 2; --jj) {
+      const int st = arg[e * P1 + jj];
+      cuts[jj - 2] = st;
+      e = st;
+    }
+  }
+}
+
+// ===========================================================================
+// K3 heuristic restarts (adjust_mode none; reading O9).
+struct HeurArgs {
+  DevTables t;
+  int p, m;
+  uint64_t seed;
+  int radius;
+  uint32_t r_lo, r_hi;
+  const int16_t* arg;
+  const int32_t* alg1;
+  unsigned int* counter;
+  unsigned long long* key;
+  int32_t* replay;
+};
+
+// Algorithm 1 on the prefix [0, c) with j stages: writes c_1..c_{j-1} (line 15).
+AP_DEV_INLINE void alg1_prefix(const int16_t* s_arg, int P1, int c, int j, int* cut) {
+  int e = c;
+  for (int jj = j; jj >= 2; --jj) {
+    const int st = s_arg[e * P1 + jj];
+    cut[jj - 1] = st;
+    e = st;
+  }
+}
+
+template <int P>
+__global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int n = A.t.n, p = A.p, m = A.m, P1 = p + 1;
+  int16_t* s_arg = reinterpret_cast<int16_t*>(smem + ((used + 15) & ~size_t(15)));
+  const int narg = (n + 1) * P1;
+  int32_t* s_a1 = reinterpret_cast<int32_t*>(s_arg + ((narg + 7) & ~7));
+  uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_a1 + 32);
+  for (int e = threadIdx.x; e < narg; e += blockDim.x) s_arg[e] = A.arg[e];
+  for (int e = threadIdx.x; e < p - 1; e += blockDim.x) s_a1[e] = A.alg1[e];
+  __syncthreads();
+  BitsRef br{s_bits + threadIdx.x, (int)blockDim.x};
+  TimesRef not_{nullptr, nullptr, nullptr};
+
+  int cur[P + 1], cand[P + 1], best[P + 1], sel[P + 1];
+  unsigned long long lane_key = 0x7fffffffffffffffull;
+  const int smax = n * p;
+  int phase = 0;  // 0 need restart, 1 start evaluated next, 2 child evaluated next
+  uint32_t r = 0;
+  int64_t bestT = 0, selT = 0;
+  int curM = 0, selM = 0, steps = 0, chIdx = 0;
+
+  // child generator: idx 0 a, 1 a', 2 b, 3 b' (reading Q17)
+  auto gen_child = [&](int idx, int i) -> bool {
+    const int size_i = cur[i + 1] - cur[i];
+    if (size_i < 2) return false;
+#pragma unroll
+    for (int x = 0; x <= P; ++x) cand[x] = cur[x];
+    if (idx <= 1) {
+      cand[i] += 1;  // first block of stage i -> stage i-1
+      if (idx == 0) return true;
+      if (i - 1 < 1) return false;
+      alg1_prefix(s_arg, P1, cand[i - 1], i - 1, cand);
+      bool diff = false;
+      for (int x = 1; x < i - 1; ++x) diff = diff || (cand[x] != cur[x]);
+      return diff;
+    }
+    if (i > p - 2) return false;
+    cand[i + 1] -= 1;  // last block of stage i -> stage i+1
+    if (idx == 2) return true;
+    alg1_prefix(s_arg, P1, cand[i], i, cand);
+    bool diff = false;
+    for (int x = 1; x < i; ++x) diff = diff || (cand[x] != cur[x]);
+    return diff;
+  };
+
+  for (;;) {
+    if (phase == 0) {
+      r = atomicAdd(A.counter, 1u) + A.r_lo;
+      if (r >= A.r_hi) break;
+      // restart start: Alg. 1 (r = 0) or the seeded perturbation (reading Q21)
+      cand[0] = 0;
+#pragma unroll
+      for (int x = 1; x <= P; ++x) cand[x] = n;
+      int prev = 0;
+      for (int x = 1; x <= p - 1; ++x) {
+        int64_t v = s_a1[x - 1];
+        if (r != 0) {
+          const uint64_t u = splitmix64(A.seed ^ ((uint64_t)r << 32) ^ (uint64_t)x);
+          v += (int64_t)(u % (uint64_t)(2 * A.radius + 1)) - A.radius;
+          v = v < prev + 1 ? prev + 1 : v;
+          v = v > n - (p - x) ? n - (p - x) : v;
+        }
+        cand[x] = (int)v;
+        prev = (int)v;
+      }
+      phase = 1;
+    }
+    // ---- simulate cand (k = 1) with its master stage
+    int cc[P + 1];
+#pragma unroll
+    for (int x = 0; x <= P; ++x) cc[x] = cand[x];
+    int64_t F[P], B[P], C[P];
+    stage_costs<P>(T, p, cc, F, B, C);
+    uint32_t pb[P];
+    const int64_t Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
+    int len;
+    const int Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+    bool do_step = false, finish = false;
+    if (phase == 1) {
+      curM = Mc;
+      bestT = Tc;
+      for (int x = 0; x <= p; ++x) {
+        cur[x] = cand[x];
+        best[x] = cand[x];
+      }
+      steps = 0;
+      do_step = true;
+    } else {
+      if (Tc < bestT) {
+        bestT = Tc;
+        for (int x = 0; x <= p; ++x) best[x] = cand[x];
+      }
+      if (Mc <= curM && Tc < selT) {
+        selT = Tc;
+        selM = Mc;
+        for (int x = 0; x <= p; ++x) sel[x] = cand[x];
+      }
+      bool found = false;
+      for (int idx = chIdx + 1; idx <= 3 && !found; ++idx)
+        if (gen_child(idx, curM)) {
+          chIdx = idx;
+          found = true;
+        }
+      if (!found) {
+        if (selT == INT64_MAX) {
+          finish = true;
+        } else {
+          for (int x = 0; x <= p; ++x) cur[x] = sel[x];
+          curM = selM;
+          do_step = true;
+        }
+      }
+    }
+    if (do_step) {
+      if (curM == 0 || steps >= smax) {
+        finish = true;
+      } else {
+        ++steps;
+        selT = INT64_MAX;
+        bool found = false;
+        for (int idx = 0; idx <= 3 && !found; ++idx)
+          if (gen_child(idx, curM)) {
+            chIdx = idx;
+            found = true;
+          }
+        if (!found) finish = true;
+        else phase = 2;
+      }
+    }
+    if (finish) {
+      if (bestT < (1ll << 43)) lane_key = min(lane_key, ((unsigned long long)bestT << 20) | r);
+      if (A.replay)
+        for (int x = 1; x <= p - 1; ++x) A.replay[x - 1] = best[x];
+      phase = 0;
+    }
+  }
+  block_min_atomic(lane_key, A.key);
+}
+
+// ===========================================================================
+// Critical path with times (single candidate; thread 0).
+struct CpathArgs {
+  DevTables t;
+  int p, m, k;
+  const int32_t* cuts;
+  OpRec* ops;
+  int cap;
+  int32_t* len_master;  // [0] = len, [1] = master
+  int64_t* T;
+  uint32_t* bits;
+  int64_t* finF;
+  int64_t* finB;
+  int64_t* finP;
+  int* order;  // path scratch: encoded ops sink -> source
+};
+
+template <int P>
+__global__ void k_cpath(CpathArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  if (threadIdx.x != 0) return;
+  const int p = A.p, m = A.m, k = A.k, n = A.t.n;
+  int c[P + 1];
+  if (!load_cuts<P>(A.cuts, p, n, c)) {
+    A.len_master[0] = -1;
+    return;
+  }
+  int64_t F[P], B[P], C[P];
+  stage_costs<P>(T, p, c, F, B, C);
+  uint32_t pb[P];
+  BitsRef br{A.bits, 1};
+  TimesRef tr{A.finF, A.finB, A.finP};
+  const int64_t Tc = sim_exact<P, 2>(p, m, k, F, B, C, br, pb, tr);
+  int len = 0;
+  int* order = A.order;
+  int cnt = 0;
+  const int master = backtrack_master<P>(p, m, k, br, pb, &len, [&](int kind, int x, int j, int q) {
+    // kind:1 | x:5 | q:5 | j:20 bits (m <= 2^20, p <= 32, k <= 16)
+    order[cnt++] = (int)((((uint32_t)kind << 10 | (uint32_t)x << 5 | (uint32_t)q) << 20) | (uint32_t)j);
+  });
+  A.len_master[0] = len;
+  A.len_master[1] = master;
+  *A.T = Tc;
+  if (len > A.cap) return;
+  const int W0 = min(p - 1, m);
+  for (int e = 0; e < len; ++e) {
+    const uint32_t code = (uint32_t)order[len - 1 - e];
+    const int j = (int)(code & ((1u << 20) - 1));
+    const int q = (int)((code >> 20) & 31u);
+    const int x = (int)((code >> 25) & 31u);
+    const int kind = (int)(code >> 30);
+    int64_t fin = 0, cost = 0;
+    int xx = 0;
+#pragma unroll
+    for (int s = 0; s < P; ++s) xx = (s == x) ? s : xx;
+    int64_t Fx = 0, Bx = 0;
+#pragma unroll
+    for (int s = 0; s < P; ++s)
+      if (s == x) {
+        Fx = F[s];
+        Bx = B[s];
+      }
+    const int wx = min(p - 1 - x, m);
+    if (kind == 1) {
+      fin = A.finB[(j + W0) * P + x];
+      cost = Bx;
+    } else if (j == 0) {
+      fin = A.finP[x * kMaxK + q];
+      cost = (q < k - 1) ? Fx / k : Fx - (int64_t)(k - 1) * (Fx / k);
+    } else {
+      fin = A.finF[(j - wx + W0) * P + x];
+      cost = Fx;
+    }
+    (void)xx;
+    OpRec o;
+    o.stage = x;
+    o.kind = kind;
+    o.microbatch = j;
+    o.piece = q;
+    o.start_ns = fin - cost;
+    o.end_ns = fin;
+    A.ops[e] = o;
+  }
+}
+
+__global__ void k_unrank(DevTables t, int p, uint64_t rank, int32_t* cuts) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  const int n = t.n;
+  uint64_t rr = rank;
+  int prev = 0;
+  for (int x = 1; x <= p - 1; ++x) {
+    int v = prev + 1;
+    for (;;) {
+      const uint64_t cnt = binom_at(t.binom, n - 1 - v, p - 1 - x);
+      if (rr >= cnt) {
+        rr -= cnt;
+        ++v;
+      } else {
+        break;
+      }
+    }
+    cuts[x - 1] = v;
+    prev = v;
+  }
+}
+
+// ===========================================================================
+// Launchers.
+static int pick_P(int p) { return p <= 2 ? 2 : p <= 4 ? 4 : p <= 8 ? 8 : p <= 16 ? 16 : 32; }
+
+int num_sms(int device) {
+  int v = 0;
+  cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, device);
+  return v;
+}
+
+static cudaError_t set_smem(const void* fn, size_t bytes) {
+  if (bytes > 48 * 1024)
+    return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)bytes);
+  return cudaSuccess;
+}
+
+cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, int64_t* value,
+                        cudaStream_t s) {
+  const size_t smem = ((tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15)) +
+                      (size_t)(t.n + 1) * (p + 1) * 8;
+  cudaError_t e = set_smem((const void*)k_alg1, smem);
+  if (e != cudaSuccess) return e;
+  k_alg1<<<1, 256, smem, s>>>(t, p, arg, cuts, value);
+  return cudaGetLastError();
+}
+
+template <int P>
+static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
+  EvalArgs A = A0;
+  const size_t base = (tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15);
+  int threads = 128;
+  size_t smem = base;
+  if (A.master) {
+    const int rows = A.m + min(A.p - 1, A.m);
+    const size_t per = (size_t)rows * BitsLayout<P>::WPR * 4;
+    const size_t budget = 200 * 1024 - base;
+    if (per * 32 > budget) {
+      // bits in global scratch: caller provided A.gbits
+      if (!A.gbits) return cudaErrorInvalidValue;
+    } else {
+      A.gbits = nullptr;
+      { const size_t cap = (budget / per) / 32 * 32; threads = (int)(cap < 128 ? cap : 128); }
+      smem = base + per * threads;
+    }
+  }
+  cudaError_t e = set_smem((const void*)k_eval<P>, smem);
+  if (e != cudaSuccess) return e;
+  const int64_t blocks = (A.count + threads - 1) / threads;
+  if (blocks > 0) {
+    k_eval<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+    if (launches) ++*launches;
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_eval(const DevTables& t, int p, int m, const int32_t* cuts, int cuts_stride,
+                        const int32_t* kptr, int k_const, int k_iota, int64_t count,
+                        int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches) {
+  EvalArgs A{t, p, m, cuts, cuts_stride, kptr, k_const, k_iota, count, time_ns, master, nullptr};
+  uint32_t* gbits = nullptr;
+  if (master) {
+    const int rows = m + min(p - 1, m);
+    const int P = pick_P(p);
+    const size_t per = (size_t)rows * (P <= 16 ? 1 : 2) * 4;
+    const size_t base = (tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15);
+    if (per * 32 > 200 * 1024 - base) {
+      cudaError_t e = cudaMallocAsync((void**)&gbits, per * (size_t)count + 16, s);
+      if (e != cudaSuccess) return e;
+      A.gbits = gbits;
+    }
+  }
+  cudaError_t e;
+  switch (pick_P(p)) {
+    case 2: e = eval_P<2>(A, s, launches); break;
+    case 4: e = eval_P<4>(A, s, launches); break;
+    case 8: e = eval_P<8>(A, s, launches); break;
+    case 16: e = eval_P<16>(A, s, launches); break;
+    default: e = eval_P<32>(A, s, launches); break;
+  }
+  if (gbits) cudaFreeAsync(gbits, s);
+  return e;
+}
+
+template <int P, typename V>
+static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int dev) {
+  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n) + (size_t)(3 * (A.t.n + 1) + 4) * sizeof(V);
+  const void* fn = (const void*)k_sweep_exact<P, V>;
+  cudaError_t e = set_smem(fn, smem);
+  if (e != cudaSuccess) return e;
+  const int threads = 256;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sweep_exact<P, V>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  const uint64_t nr = A.rank_hi - A.rank_lo;
+  const uint64_t target = (uint64_t)num_sms(dev) * occ * threads;
+  A.chunk = (nr + target - 1) / target;
+  if (A.chunk == 0) A.chunk = 1;
+  const uint64_t nthreads = (nr + A.chunk - 1) / A.chunk;
+  const uint64_t blocks = (nthreads + threads - 1) / threads;
+  k_sweep_exact<P, V><<<(unsigned)blocks, threads, smem, s>>>(A);
+  sp->blocks = (int)blocks;
+  sp->threads = threads;
+  sp->chunk = A.chunk;
+  return cudaGetLastError();
+}
+
+template <int P>
+static cudaError_t sweep_generic_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int dev) {
+  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n);
+  const void* fn = (const void*)k_sweep_generic<P>;
+  cudaError_t e = set_smem(fn, smem);
+  if (e != cudaSuccess) return e;
+  const int threads = 128;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sweep_generic<P>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  const uint64_t nr = A.rank_hi - A.rank_lo;
+  const uint64_t target = (uint64_t)num_sms(dev) * occ * threads;
+  A.chunk = (nr + target - 1) / target;
+  if (A.chunk == 0) A.chunk = 1;
+  const uint64_t nthreads = (nr + A.chunk - 1) / A.chunk;
+  const uint64_t blocks = (nthreads + threads - 1) / threads;
+  k_sweep_generic<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+  sp->blocks = (int)blocks;
+  sp->threads = threads;
+  sp->chunk = A.chunk;
+  return cudaGetLastError();
+}
+
+#define AP_EXACT_CASE(PP)                                                   \
+  case PP:                                                                  \
+    return want_u32 ? sweep_exact_P<PP, uint32_t>(A, s, sp, dev)            \
+                    : sweep_exact_P<PP, uint64_t>(A, s, sp, dev);
+
+static cudaError_t sweep_exact_dispatch(int p, int want_u32, const SweepArgs& A, cudaStream_t s,
+                                        SweepPlan* sp, int dev) {
+  switch (p) {
+    AP_EXACT_CASE(1)
+    AP_EXACT_CASE(2)
+    AP_EXACT_CASE(3)
+    AP_EXACT_CASE(4)
+    AP_EXACT_CASE(5)
+    AP_EXACT_CASE(6)
+    AP_EXACT_CASE(7)
+    AP_EXACT_CASE(8)
+    AP_EXACT_CASE(10)
+    AP_EXACT_CASE(12)
+    AP_EXACT_CASE(16)
+    default: return cudaErrorNotSupported;
+  }
+}
+
+bool has_exact(int p) {
+  return (p >= 1 && p <= 8) || p == 10 || p == 12 || p == 16;
+}
+
+cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
+                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int force_generic,
+                         unsigned long long* key, cudaStream_t s, SweepPlan* sp) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  k_init_key<<<1, 1, 0, s>>>(key);
+  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key};
+  const bool exact = has_exact(p) && m >= p && !force_generic;
+  sp->exact_p = exact ? 1 : 0;
+  sp->fast_u32 = (exact && want_u32) ? 1 : 0;
+  if (exact) return sweep_exact_dispatch(p, sp->fast_u32, A, s, sp, dev);
+  switch (pick_P(p)) {
+    case 2: return sweep_generic_P<2>(A, s, sp, dev);
+    case 4: return sweep_generic_P<4>(A, s, sp, dev);
+    case 8: return sweep_generic_P<8>(A, s, sp, dev);
+    case 16: return sweep_generic_P<16>(A, s, sp, dev);
+    default: return sweep_generic_P<32>(A, s, sp, dev);
+  }
+}
+
+template <int P>
+static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev) {
+  const int threads = A.replay ? 32 : 128;
+  const int rows = A.m + min(A.p - 1, A.m);
+  const size_t narg = (size_t)(A.t.n + 1) * (A.p + 1);
+  const size_t base = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
+                      ((narg + 7) & ~size_t(7)) * 2 + 32 * 4;
+  const size_t smem = base + (size_t)rows * BitsLayout<P>::WPR * 4 * threads;
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  cudaError_t e = set_smem((const void*)k_heur<P>, smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_heur<P>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  const uint64_t R = A.r_hi - A.r_lo;
+  uint64_t blocks = (uint64_t)num_sms(dev) * occ;
+  const uint64_t need = (R + threads - 1) / threads;
+  if (blocks > need) blocks = need;
+  if (blocks < 1) blocks = 1;
+  k_heur<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, int radius,
+                             uint32_t r_lo, uint32_t r_hi, const int16_t* arg,
+                             const int32_t* alg1_cuts, unsigned int* counter,
+                             unsigned long long* key, int32_t* replay_cuts, cudaStream_t s) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  k_init_key<<<1, 1, 0, s>>>(key);
+  cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned int), s);
+  if (e != cudaSuccess) return e;
+  HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts};
+  switch (pick_P(p)) {
+    case 2: return heur_P<2>(A, s, dev);
+    case 4: return heur_P<4>(A, s, dev);
+    case 8: return heur_P<8>(A, s, dev);
+    case 16: return heur_P<16>(A, s, dev);
+    default: return heur_P<32>(A, s, dev);
+  }
+}
+
+size_t cpath_scratch_bytes(int p, int m) {
+  const int rows = m + min(p - 1, m);
+  const int P = pick_P(p);
+  const size_t ops = (size_t)p * (2 * m + kMaxK);
+  return 256 + (size_t)rows * 2 * 4 + 2 * (size_t)rows * P * 8 + (size_t)P * kMaxK * 8 +
+         ops * 4 + 64;
+}
+
+template <int P>
+static cudaError_t cpath_P(CpathArgs A, cudaStream_t s) {
+  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n);
+  cudaError_t e = set_smem((const void*)k_cpath<P>, smem);
+  if (e != cudaSuccess) return e;
+  k_cpath<P><<<1, 32, smem, s>>>(A);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t* cuts, OpRec* ops,
+                         int cap, int32_t* len_master, int64_t* T, void* scratch,
+                         cudaStream_t s) {
+  const int rows = m + min(p - 1, m);
+  const int P = pick_P(p);
+  unsigned char* b = reinterpret_cast<unsigned char*>(scratch);
+  CpathArgs A;
+  A.t = t;
+  A.p = p;
+  A.m = m;
+  A.k = k;
+  A.cuts = cuts;
+  A.ops = ops;
+  A.cap = cap;
+  A.len_master = len_master;
+  A.T = T;
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    void* r = b + off;
+    off += (bytes + 255) & ~size_t(255);
+    return r;
+  };
+  A.bits = reinterpret_cast<uint32_t*>(take((size_t)rows * 2 * 4));
+  A.finF = reinterpret_cast<int64_t*>(take((size_t)rows * P * 8));
+  A.finB = reinterpret_cast<int64_t*>(take((size_t)rows * P * 8));
+  A.finP = reinterpret_cast<int64_t*>(take((size_t)P * kMaxK * 8));
+  A.order = reinterpret_cast<int*>(take((size_t)p * (2 * m + kMaxK) * 4));
+  switch (P) {
+    case 2: return cpath_P<2>(A, s);
+    case 4: return cpath_P<4>(A, s);
+    case 8: return cpath_P<8>(A, s);
+    case 16: return cpath_P<16>(A, s);
+    default: return cpath_P<32>(A, s);
+  }
+}
+
+cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,
+                          cudaStream_t s) {
+  k_unrank<<<1, 32, 0, s>>>(t, p, rank, cuts);
+  return cudaGetLastError();
+}
+
+}  // namespace apk

@@ -1,0 +1,64 @@
+// ap_launch.h -- internal interface between the C-ABI host layer (ap_host.cu) and
+// the kernels (ap_kernels.cu).  Not part of the public ABI.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace apk {
+
+struct DevTables {
+  const int64_t* tab;     // [f | b | comm], 3*npad int64, 16-B aligned (TMA source)
+  const uint64_t* binom;  // C(a, b) for a in [0, n], b in [0, 32], saturating
+  int n;
+  int npad;
+};
+
+// Algorithm 1 on the device: arg table int16[(n+1)*(p+1)],
+// the Alg.-1 cut vector int32[p-1] and its value.
+cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, int64_t* value,
+                        cudaStream_t s);
+
+// Generic exact evaluation of `count` candidates.  cuts_stride = p-1 (batch) or 0
+// (all rows share one cut vector).  k source: kptr if non-null, else k_iota ? row+1
+// : k_const.  master may be null.  Invalid rows -> time -1, master -1.
+cudaError_t launch_eval(const DevTables& t, int p, int m, const int32_t* cuts, int cuts_stride,
+                        const int32_t* kptr, int k_const, int k_iota, int64_t count,
+                        int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches);
+
+struct SweepPlan {
+  int fast_u32;   // exact u32 saturating sweep
+  int exact_p;    // kernel specialised to this p
+  int blocks, threads;
+  uint64_t chunk;
+};
+// Exhaustive sweep of ranks [rank_lo, rank_hi) x k in [k_lo, k_hi].  S = T_ref + 1:
+// a candidate with T >= S can never win.  Writes INT64_MAX first, then atomicMin.
+cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
+                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int force_generic,
+                         unsigned long long* key, cudaStream_t s, SweepPlan* plan_out);
+
+// Heuristic restarts [r_lo, r_hi); key = min (T << 20 | r).  replay_cuts (int32[p-1])
+// non-null: single-restart replay writing that restart's best cut vector.
+cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, int radius,
+                             uint32_t r_lo, uint32_t r_hi, const int16_t* arg,
+                             const int32_t* alg1_cuts, unsigned int* counter,
+                             unsigned long long* key, int32_t* replay_cuts, cudaStream_t s);
+
+struct OpRec {
+  int32_t stage, kind, microbatch, piece;
+  int64_t start_ns, end_ns;
+};
+// Critical path of one candidate: ops (source -> sink) into `ops` (cap entries),
+// len, master, T.  scratch: device bytes >= cpath_scratch_bytes(p, m).
+size_t cpath_scratch_bytes(int p, int m);
+cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t* cuts, OpRec* ops,
+                         int cap, int32_t* len_master, int64_t* T, void* scratch,
+                         cudaStream_t s);
+
+// Decode helper: unrank lex rank -> cut vector int32[p-1].
+cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,
+                          cudaStream_t s);
+
+int num_sms(int device);
+
+}  // namespace apk

@@ -1,0 +1,74 @@
+"""Multi-GPU search orchestration (one process per GPU, torch.distributed/NCCL).
+
+The candidate space is sharded by contiguous lex-rank (or restart) ranges
+``[floor(g*N/G), floor((g+1)*N/G))`` -- SURVEY.md §8e.  Each rank writes one packed
+int64 key on its GPU; ONE ``all_reduce(MIN)`` of that 8-byte key over NVLink picks
+the global winner, which every rank then decodes independently (no second
+collective).  The reduction is exact because keys order lexicographically by
+(T, rank, k) / (T, restart) -- include/ap.h.
+"""
+from __future__ import annotations
+
+from typing import Optional
+
+import torch
+
+from . import (INT64_MAX, Plan, ap_count, ap_decode, ap_search_exhaustive,
+               ap_search_heuristic)
+
+
+def shard(total: int, rank: int, world: int):
+    """Contiguous [lo, hi) slice of `total` units for `rank` of `world`."""
+    return (total * rank) // world, (total * (rank + 1)) // world
+
+
+def _world():
+    import torch.distributed as dist
+    if dist.is_available() and dist.is_initialized():
+        return dist.get_rank(), dist.get_world_size(), dist
+    return 0, 1, None
+
+
+def min_allreduce_key(key: torch.Tensor, dist=None, group=None) -> torch.Tensor:
+    """In-place MIN all-reduce of the packed int64 key (no-op on one process)."""
+    if dist is not None:
+        dist.all_reduce(key, op=dist.ReduceOp.MIN, group=group)
+    return key
+
+
+def search_exhaustive(plan: Plan, p: int, m: int, k_lo: int = 1, k_hi: int = 1,
+                      group=None, decode: bool = True, stream=None) -> dict:
+    """Exact argmin over all C(n-1,p-1) partitions x k in [k_lo,k_hi], sharded over
+    the ranks of the default process group (if initialised)."""
+    rank, world, dist = _world()
+    N = ap_count(plan.n, p)
+    lo, hi = shard(N, rank, world)
+    key = torch.empty(1, dtype=torch.int64, device=f"cuda:{plan.device}")
+    if hi > lo:
+        ap_search_exhaustive(plan, p, m, k_lo, k_hi, lo, hi, key, stream=stream)
+    else:
+        key.fill_(INT64_MAX)
+    min_allreduce_key(key, dist, group)
+    kv = int(key.item())
+    out = {"key": kv, "sims": (hi - lo) * (k_hi - k_lo + 1), "total_sims": N * (k_hi - k_lo + 1),
+           "shard": (lo, hi)}
+    if decode:
+        out.update(ap_decode(plan, 0, p, m, k_lo, k_hi, key=kv))
+    return out
+
+
+def search_heuristic(plan: Plan, p: int, m: int, restarts: int, seed: int = 0x5EED,
+                     radius: int = 2, group=None, decode: bool = True, stream=None) -> dict:
+    rank, world, dist = _world()
+    lo, hi = shard(restarts, rank, world)
+    key = torch.empty(1, dtype=torch.int64, device=f"cuda:{plan.device}")
+    if hi > lo:
+        ap_search_heuristic(plan, p, m, seed, radius, lo, hi, 0, key, stream=stream)
+    else:
+        key.fill_(INT64_MAX)
+    min_allreduce_key(key, dist, group)
+    kv = int(key.item())
+    out = {"key": kv, "shard": (lo, hi)}
+    if decode:
+        out.update(ap_decode(plan, 1, p, m, seed=seed, radius=radius, key=kv))
+    return out

@@ -1,0 +1,329 @@
+"""GPU <-> oracle parity (-m gpu).  Bit-exact on every integer output.
+
+Every GPU call goes through the C ABI (libap.so via the thin binding); every
+expected value comes from oracle/ on the same seeded synth inputs.
+"""
+import math
+import os
+
+import numpy as np
+import pytest
+
+import synth
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ap():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_cluster_liulldgl22_b200 as ap
+    return ap
+
+
+def _plan(ap, f, b, a, bw):
+    return ap.ap_plan_create(f, b, a, bw, device=0)
+
+
+def _eval(ap, plan, p, m, cuts, ks, master=True):
+    import torch
+    cnt = len(cuts)
+    c = torch.tensor(np.asarray(cuts, np.int32).reshape(cnt, max(p - 1, 0)), device="cuda")
+    if p == 1:
+        c = torch.zeros((cnt, 0), dtype=torch.int32, device="cuda")
+    k = torch.tensor(np.asarray(ks, np.int32), device="cuda")
+    T = torch.empty(cnt, dtype=torch.int64, device="cuda")
+    M = torch.empty(cnt, dtype=torch.int32, device="cuda") if master else None
+    ap.ap_eval_batch(plan, p, m, c, k, T, M)
+    torch.cuda.synchronize()
+    return T.cpu().numpy(), (M.cpu().numpy() if master else None)
+
+
+# --------------------------------------------------------------------------- K2
+@pytest.mark.parametrize("kind", ["uniform", "b3f", "small", "equal", "huge", "zero"])
+def test_eval_batch_random_vs_oracle(ap, oracle_mod, kind):
+    """Random (n, p, m, k, cuts) incl. m < p-1, ties, zero costs: T and master."""
+    rng = np.random.default_rng(hash(kind) % 1000)
+    for trial in range(12):
+        n = int(rng.integers(2, 40))
+        f, b, a = synth.random_tables(trial * 7 + len(kind), n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        for p in sorted({1, 2, int(rng.integers(1, min(n, 32) + 1)), min(n, 16)}):
+            m = int(rng.choice([1, 2, 3, p - 1 if p > 1 else 1, p, p + 1, 2 * p + 3, 40]))
+            cnt = 24
+            cuts = synth.random_cuts(trial + 100 * p, n, p, cnt)
+            ks = rng.integers(1, 17, cnt)
+            T, Ms = _eval(ap, plan, p, m, cuts, ks)
+            for i in range(cnt):
+                r = M.simulate(p, m, cuts[i], k=int(ks[i]))
+                assert T[i] == r["T"], (kind, n, p, m, int(ks[i]), list(cuts[i]))
+                assert Ms[i] == r["master"], (kind, n, p, m, int(ks[i]), list(cuts[i]))
+
+
+def test_eval_batch_invalid_rows(ap):
+    import torch
+    f, b, a = synth.random_tables(1, 10)
+    plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+    cuts = torch.tensor([[3, 5, 7], [5, 3, 7], [0, 3, 7], [3, 5, 10]], dtype=torch.int32, device="cuda")
+    k = torch.tensor([1, 1, 1, 1], dtype=torch.int32, device="cuda")
+    T = torch.empty(4, dtype=torch.int64, device="cuda")
+    ap.ap_eval_batch(plan, 4, 8, cuts, k, T)
+    assert T.cpu().tolist()[1:] == [-1, -1, -1] and T.cpu().tolist()[0] > 0
+
+
+def test_table2_partitions(ap, oracle_mod):
+    """PAPER.md Table II partitions (GPT-2 345M, p=4) as named eval inputs."""
+    import json
+    doc = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "table2_gpt2_345m.json")))
+    wl = synth.config(2)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model(f, b, a, wl.link_bytes_per_s)
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    cuts = [prt["cuts"] for prt in doc["partitions"]]
+    for m in (8, 16):
+        T, Ms = _eval(ap, plan, 4, m, cuts, [1] * len(cuts))
+        for i, c in enumerate(cuts):
+            r = M.simulate(4, m, c)
+            assert (T[i], Ms[i]) == (r["T"], r["master"])
+
+
+# --------------------------------------------------------------------------- cpath
+def test_critical_path_vs_oracle(ap, oracle_mod):
+    rng = np.random.default_rng(5)
+    for trial in range(40):
+        kind = ["small", "uniform", "b3f"][trial % 3]
+        n = int(rng.integers(2, 20))
+        f, b, a = synth.random_tables(trial, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p = int(rng.integers(1, min(n, 16) + 1))
+        m = int(rng.integers(1, 12))
+        k = int(rng.integers(1, 6))
+        cuts = synth.random_cuts(trial, n, p, 1)[0]
+        g = ap.ap_critical_path(plan, p, m, k, cuts)
+        o = M.simulate(p, m, cuts, k=k, want_path=True)
+        assert g["T"] == o["T"] and g["master"] == o["master"]
+        assert g["path"] == o["path"], (n, p, m, k)
+
+
+def test_critical_path_capacity(ap):
+    f, b, a = synth.random_tables(3, 12)
+    plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+    with pytest.raises(ap.APError) as ei:
+        ap.ap_critical_path(plan, 4, 8, 1, [3, 6, 9], cap=2)
+    assert ei.value.status == 5
+
+
+# --------------------------------------------------------------------------- Alg. 1
+def test_alg1_vs_oracle(ap, oracle_mod):
+    for seed in range(30):
+        kind = ["uniform", "small", "equal"][seed % 3]
+        n = 1 + (seed * 7) % 120
+        f, b, a = synth.random_tables(seed, n, kind)
+        M = oracle_mod.Model(f, b, a, synth.link_for(kind))
+        plan = _plan(ap, f, b, a, synth.link_for(kind))
+        for p in sorted({1, min(n, 2), min(n, 7), min(n, 16), min(n, 32)}):
+            gc, gv = ap.ap_alg1(plan, p)
+            oc, ov = M.alg1(p)
+            assert list(gc) == list(oc) and gv == ov, (n, p)
+    for i in synth.ALL_CONFIGS:
+        wl = synth.config(i)
+        f, b, a = wl.arrays()
+        plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+        oc, ov = oracle_mod.Model.from_workload(wl).alg1(wl.p)
+        gc, gv = ap.ap_alg1(plan, wl.p)
+        assert list(gc) == list(oc) and gv == ov
+
+
+# --------------------------------------------------------------------------- K1
+def _search(ap, plan, p, m, k_lo, k_hi, lo=None, hi=None):
+    import torch
+    N = ap.ap_count(plan.n, p)
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    ap.ap_search_exhaustive(plan, p, m, k_lo, k_hi, 0 if lo is None else lo, N if hi is None else hi, key)
+    torch.cuda.synchronize()
+    return int(key.item())
+
+
+@pytest.mark.parametrize("mode", ["", "int64", "generic"])
+def test_exhaustive_small_random_vs_oracle(ap, oracle_mod, mode, monkeypatch):
+    if mode:
+        monkeypatch.setenv("AP_SWEEP", mode)
+    rng = np.random.default_rng(11)
+    for trial in range(14):
+        kind = ["uniform", "b3f", "small", "equal"][trial % 4]
+        n = int(rng.integers(3, 16))
+        f, b, a = synth.random_tables(trial, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p = int(rng.integers(1, min(n, 6) + 1))
+        m = int(rng.choice([1, 2, p, p + 3, 12]))
+        k_lo = int(rng.integers(1, 3)); k_hi = k_lo + int(rng.integers(0, 4))
+        key = _search(ap, plan, p, m, k_lo, k_hi)
+        res = ap.ap_decode(plan, 0, p, m, k_lo, k_hi, key=key)
+        o = M.exhaustive(p, m, k_lo, k_hi)
+        assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"]), (n, p, m, k_lo, k_hi, mode)
+        assert res["cuts"] == [int(x) for x in o["cuts"]]
+        assert res["master"] == M.simulate(p, m, o["cuts"], k=o["k"])["master"]
+
+
+@pytest.mark.parametrize("cfg", [1, 2])
+def test_exhaustive_configs_full_vs_oracle(ap, oracle_mod, cfg):
+    """C1 and C2 exactly: full oracle brute force vs the GPU sweep + decode."""
+    wl = synth.config(cfg)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model.from_workload(wl)
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    key = _search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
+    info = ap.ap_last_launch()
+    res = ap.ap_decode(plan, 0, wl.p, wl.m, wl.k_lo, wl.k_hi, key=key)
+    o = M.exhaustive_parallel(wl.p, wl.m, wl.k_lo, wl.k_hi)
+    assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+    assert info["fast_u32"] == 1 and info["exact_p"] == 1
+    # k = 1 subproblem of C2 as well
+    if cfg == 2:
+        key = _search(ap, plan, 4, 16, 1, 1)
+        res = ap.ap_decode(plan, 0, 4, 16, 1, 1, key=key)
+        assert (res["time_ns"], res["rank"]) == (89891590, 12221)
+
+
+@pytest.mark.parametrize("cfg", [3, 4])
+def test_exhaustive_big_configs_vs_oracle_bnb(ap, oracle_mod, cfg):
+    """C3 / C4 at full size, in the bench's launch configuration: the GPU argmin
+    equals the oracle's exact argmin (its LB-skipping enumeration, same order)."""
+    wl = synth.config(cfg)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model.from_workload(wl)
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    key = _search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
+    info = ap.ap_last_launch()
+    assert info["fast_u32"] == 1
+    res = ap.ap_decode(plan, 0, wl.p, wl.m, wl.k_lo, wl.k_hi, key=key)
+    o = M.exhaustive_bnb(wl.p, wl.m, wl.k_lo, wl.k_hi)
+    assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+    assert res["cuts"] == [int(x) for x in o["cuts"]]
+
+
+def test_exhaustive_sampled_ranks_big(ap, oracle_mod):
+    """C4 sampled: the GPU's argmin over many tiny rank windows (bench kernel,
+    u32 path) equals the oracle's brute force over the same windows."""
+    wl = synth.config(4)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model.from_workload(wl)
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    N = ap.ap_count(wl.n, wl.p)
+    rng = np.random.default_rng(4)
+    for lo in rng.integers(0, N - 40, 12):
+        lo = int(lo)
+        key = _search(ap, plan, wl.p, wl.m, 1, 8, lo, lo + 40)
+        o = M.exhaustive(wl.p, wl.m, 1, 8, lo, lo + 40)
+        T_ref = ap.ap_last_launch()["t_ref"]
+        if o["T"] > T_ref:
+            assert key == (1 << 63) - 1
+        else:
+            res = ap.ap_decode(plan, 0, wl.p, wl.m, 1, 8, key=key)
+            assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+
+
+def test_fake_sharding_equals_single(ap, oracle_mod):
+    """G shards run one after another and min-reduced == the 1-shard key, for
+    several G (the multi-GPU decomposition of SURVEY §8e, on one GPU)."""
+    wl = synth.config(2)
+    f, b, a = wl.arrays()
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    from paper_conf_cluster_liulldgl22_b200.search import shard
+    N = ap.ap_count(wl.n, wl.p)
+    full = _search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
+    for G in (2, 3, 8, 13):
+        keys = []
+        for g in range(G):
+            lo, hi = shard(N, g, G)
+            keys.append(_search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi, lo, hi))
+        assert min(keys) == full
+
+
+# --------------------------------------------------------------------------- K3
+def test_heuristic_random_vs_oracle(ap, oracle_mod):
+    rng = np.random.default_rng(8)
+    import torch
+    for trial in range(10):
+        n = int(rng.integers(6, 30))
+        f, b, a = synth.random_tables(trial, n, ["b3f", "uniform", "small"][trial % 3])
+        bw = synth.LINK_BYTES_PER_S if trial % 3 != 2 else 10**9
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p = int(rng.integers(2, min(n, 9) + 1))
+        m = int(rng.integers(1, 3 * p))
+        R = 300
+        key = torch.empty(1, dtype=torch.int64, device="cuda")
+        ap.ap_search_heuristic(plan, p, m, 0x5EED, 2, 0, R, 0, key)
+        torch.cuda.synchronize()
+        kv = int(key.item())
+        o = M.heuristic(p, m, 0x5EED, 2, 0, R)
+        assert (kv >> 20, kv & ((1 << 20) - 1)) == (o["T"], o["restart"]), (n, p, m)
+        res = ap.ap_decode(plan, 1, p, m, seed=0x5EED, radius=2, key=kv)
+        assert res["cuts"] == [int(x) for x in o["cuts"]] and res["time_ns"] == o["T"]
+        # per-restart: single-restart ranges give each restart's own T
+        for r in (0, 1, 7):
+            ap.ap_search_heuristic(plan, p, m, 0x5EED, 2, r, r + 1, 0, key)
+            torch.cuda.synchronize()
+            assert int(key.item()) >> 20 == M.heuristic_restart(p, m, 0x5EED, 2, r)["T"]
+
+
+def test_heuristic_C2_and_C5(ap, oracle_mod):
+    """C5 at full size: all 65 536 restarts, GPU winner == oracle winner (the oracle
+    runs the same restarts on the host cores)."""
+    import torch
+    for cfg, R in ((2, 4096), (5, 65536)):
+        wl = synth.config(cfg)
+        f, b, a = wl.arrays()
+        M = oracle_mod.Model.from_workload(wl)
+        plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+        key = torch.empty(1, dtype=torch.int64, device="cuda")
+        ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, R, 0, key)
+        torch.cuda.synchronize()
+        kv = int(key.item())
+        o = M.heuristic_parallel(wl.p, wl.m, wl.seed, wl.radius, 0, R)
+        assert (kv >> 20, kv & ((1 << 20) - 1)) == (o["T"], o["restart"])
+        res = ap.ap_decode(plan, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=kv)
+        assert res["cuts"] == [int(x) for x in o["cuts"]]
+        if cfg == 5:
+            assert o["T"] <= 430480412  # restart 0 alone reaches this
+
+
+# --------------------------------------------------------------------------- slicer
+def test_slice_sweep_vs_oracle(ap, oracle_mod):
+    for cfg in (1, 2, 4, 5):
+        wl = synth.config(cfg)
+        f, b, a = wl.arrays()
+        M = oracle_mod.Model.from_workload(wl)
+        plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+        cuts, _ = M.alg1(wl.p)
+        T, bk = ap.ap_slice_sweep(plan, wl.p, wl.m, cuts, 16)
+        oT, obk = M.slice_sweep(wl.p, wl.m, cuts, 16)
+        assert list(T) == list(oT) and bk == obk
+
+
+def test_overflow_guard_and_errors(ap):
+    import torch
+    big = np.full(4, 1 << 58, np.int64)
+    plan = ap.ap_plan_create(big, big, np.zeros(4, np.int64), 10**9)
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    with pytest.raises(ap.APError) as ei:
+        ap.ap_search_exhaustive(plan, 2, 64, 1, 1, 0, 3, key)
+    assert ei.value.status == 2
+    f, b, a = synth.random_tables(1, 10)
+    plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+    with pytest.raises(ap.APError) as ei:
+        ap.ap_search_exhaustive(plan, 4, 8, 1, 1, 5, 5, key)
+    assert ei.value.status == 1
+    with pytest.raises(ap.APError):
+        ap.ap_search_exhaustive(plan, 11, 8, 1, 1, 0, 1, key)
+    with pytest.raises(ap.APError):
+        ap.ap_decode(plan, 0, 4, 8, 1, 1, key=(1 << 63) - 1)

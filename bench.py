@@ -1,0 +1,438 @@
+#!/usr/bin/env python
+"""Bench: candidate schedules simulated/s and time-to-optimal-plan (BASELINE.json).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 4] [--impl ours|reference]
+
+One step = one pass of the whole hot path over the
+workload: Algorithm 1 + T_ref, the exhaustive sweep of this rank's shard of all
+C(n-1,p-1) partitions x k (every pair fully simulated), the per-GPU argmin, ONE NCCL
+all_reduce(MIN) of the packed 8-byte key (N>1), decode (unrank + critical path +
+master stage) and the Slicer sweep of the winner.  Default workload = BASELINE.json
+configs[3] (C4, GPT-3-2.7B-shaped, n=66, p=8, m=64, k in 1..8: 5.57e9 simulations),
+the largest exhaustive config.  Multi-GPU: the rank space is split across ranks
+("strong" scaling: total work fixed); value = all simulations / max-over-ranks time.
+
+Rank 0 prints ONE JSON line.  See DESIGN.md §7 for every field.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import synth  # noqa: E402
+
+METRIC = "candidate schedules simulated/sec"
+MEASURED = os.path.join(ROOT, "MEASURED_PEAKS.json")
+
+
+def _env_rank():
+    return (int(os.environ.get("RANK", 0)), int(os.environ.get("LOCAL_RANK", 0)),
+            int(os.environ.get("WORLD_SIZE", 1)))
+
+
+def _peaks():
+    try:
+        with open(MEASURED) as fh:
+            d = json.load(fh)
+        return d, "measured"
+    except Exception:
+        return {"sm_max_mhz": 1965.0}, "fallback"
+
+
+def int_peak_ops(sm_mhz: float, sms: int = 148) -> float:
+    """Integer ALU roofline: 4 SMSPs x 32 lanes issue one warp
+    instruction per clock per SMSP = 128 int32 lanes/clk/SM, split between the alu
+    pipe (VIMNMX, 64/clk) and the fma pipe (VIADD/IMAD, 64/clk)."""
+    return sms * 128 * sm_mhz * 1e6
+
+
+def ops_per_sim(p: int, m: int, k: int) -> int:
+    """Algorithmic int32 ops of one simulation: one add per op of
+    the task DAG (its weight, receive comm included) plus one max per DISTINCT pair
+    of predecessors.  B(x,y) and F(x+1, y+w_x) have the same two predecessors
+    (B(x+1,y), F(x,y+w_x)) wherever w_x = w_{x+1}+1, so that max is counted once.
+    The naive count of SURVEY.md §8d (2 ops per op) is ops_per_sim_naive."""
+    nops = p * (2 * m + k - 1)
+    w = [min(p - 1 - x, m) for x in range(p)]
+    two_pred = (p - 1) * (m - 1 + k - 1) + (p - 1) * m
+    shared = sum(m - w[x] for x in range(p - 1) if w[x] == w[x + 1] + 1)
+    return nops + two_pred - shared
+
+
+def ops_per_sim_naive(p: int, m: int, k: int) -> int:
+    """2pm + (k-1)p max-plus ops, one max + one add each."""
+    return 2 * (2 * p * m + (k - 1) * p)
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled DURING the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap,power.draw")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.idx), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self._t = threading.Thread(target=self._read, daemon=True)
+            self._t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for ln in self.proc.stdout:
+            self.lines.append(ln.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [x.strip() for x in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0])); smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "samples": len(sm), "reasons": sorted(reasons)}
+
+
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+# ----------------------------------------------------------------------------- oracle
+def oracle_rate(wl, budget_s: float = 24.0, threads: int = 0):
+    """The oracle as it stands (plain C DAG simulator, brute force in lex order) on
+    the host cores, on a bounded sample of the workload: contiguous rank windows
+    starting at evenly spaced ranks, all k each.  Returns sims/s."""
+    import oracle
+    M = oracle.Model.from_workload(wl)
+    N = oracle.count(wl.n, wl.p)
+    threads = threads or os.cpu_count() or 1
+    K = wl.k_hi - wl.k_lo + 1
+    # calibrate one thread on a small window
+    t0 = time.perf_counter()
+    M.exhaustive(wl.p, wl.m, wl.k_lo, wl.k_hi, 0, min(N, 64))
+    per_sim = (time.perf_counter() - t0) / (min(N, 64) * K)
+    per_thread = max(1, int(budget_s / per_sim / K / threads))
+    starts = [int(N * i / threads) for i in range(threads)]
+    from concurrent.futures import ThreadPoolExecutor
+    t0 = time.perf_counter()
+    with ThreadPoolExecutor(threads) as ex:
+        res = list(ex.map(lambda s: M.exhaustive(wl.p, wl.m, wl.k_lo, wl.k_hi, s,
+                                                 min(N, s + per_thread)), starts))
+    dt = time.perf_counter() - t0
+    sims = sum(r["sims"] for r in res)
+    return {"value": sims / dt, "unit": "sims/s", "cores": threads, "kind": "oracle",
+            "sample": f"{sims} simulations: {threads} contiguous lex-rank windows of "
+                      f"{per_thread} partitions x k in [{wl.k_lo},{wl.k_hi}] at evenly spaced "
+                      f"start ranks of the {N}-partition space ({dt:.1f} s wall)",
+            "cpu": cpu_model()}
+
+
+def run_reference(args):
+    rank, local, world = _env_rank()
+    if rank != 0:
+        return 0
+    wl = synth.config(args.config)
+    steps = []
+    for i in range(args.warmup + args.steps):
+        r = oracle_rate(wl, budget_s=args.ref_budget)
+        if i >= args.warmup:
+            steps.append(r)
+    val = statistics.median(r["value"] for r in steps)
+    cb = dict(steps[-1])
+    cb["value"] = val
+    N = synth_count(wl)
+    total = N * (wl.k_hi - wl.k_lo + 1)
+    out = {"impl": "reference", "metric": METRIC, "value": val, "unit": "sims/s",
+           "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+           "ms_per_step": 1e3 * statistics.median(
+               int(r["sample"].split()[0]) / r["value"] for r in steps),
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+           "dtype": "int64", "data": "synthetic",
+           "config": {"workload": wl.name, "n": wl.n, "p": wl.p, "m": wl.m,
+                      "k": [wl.k_lo, wl.k_hi], "search": wl.search, "total_sims": total,
+                      "extrapolated_time_to_plan_s": total / val},
+           "cpu_baseline": cb,
+           "e2e": {"value": val, "unit": "sims/s", "h2d_bytes_per_step": 0,
+                   "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+    return 0
+
+
+def synth_count(wl):
+    from math import comb
+    return comb(wl.n - 1, wl.p - 1)
+
+
+# ----------------------------------------------------------------------------- ours
+def main():
+    ap_ = argparse.ArgumentParser()
+    ap_.add_argument("--gpus", type=int, default=1)
+    ap_.add_argument("--steps", type=int, default=10)
+    ap_.add_argument("--warmup", type=int, default=3)
+    ap_.add_argument("--config", type=int, default=4)
+    ap_.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap_.add_argument("--no-cpu-baseline", action="store_true")
+    ap_.add_argument("--no-secondary", action="store_true")
+    ap_.add_argument("--ref-budget", type=float, default=8.0)
+    args = ap_.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cluster_liulldgl22_b200 as ap
+    from paper_conf_cluster_liulldgl22_b200.search import shard
+
+    rank, local, world = _env_rank()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    peaks, peak_src = _peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    sms = torch.cuda.get_device_properties(local).multi_processor_count
+
+    wl = synth.config(args.config)
+    f, b, a = wl.arrays()
+    K = wl.k_hi - wl.k_lo + 1
+    plan = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=local)
+    N = ap.ap_count(wl.n, wl.p)
+    lo, hi = shard(N, rank, world)
+    total_sims = N * K
+    my_ops = (hi - lo) * sum(ops_per_sim(wl.p, wl.m, k) for k in range(wl.k_lo, wl.k_hi + 1))
+    my_ops_naive = (hi - lo) * sum(ops_per_sim_naive(wl.p, wl.m, k)
+                                   for k in range(wl.k_lo, wl.k_hi + 1))
+    key = torch.empty(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(256 * 1024 * 1024, dtype=torch.uint8, device=dev)  # > 126 MB L2
+
+    def step(pl):
+        """One time-to-optimal-plan pass through the public C-ABI binding."""
+        if hi > lo:
+            ap.ap_search_exhaustive(pl, wl.p, wl.m, wl.k_lo, wl.k_hi, lo, hi, key)
+        else:
+            key.fill_(ap.INT64_MAX)
+        if world > 1:
+            dist.all_reduce(key, op=dist.ReduceOp.MIN)
+        kv = int(key.item())
+        res = ap.ap_decode(pl, 0, wl.p, wl.m, wl.k_lo, wl.k_hi, key=kv)
+        Tk, bk = ap.ap_slice_sweep(pl, wl.p, wl.m, res["cuts"], wl.k_hi)
+        return res, Tk, bk
+
+    for _ in range(args.warmup):
+        res, Tk, bk = step(plan)
+    # ------------------------------------------------------------- timed region
+    gpu_idx = local
+    cvd = os.environ.get("CUDA_VISIBLE_DEVICES")
+    if cvd:
+        try:
+            gpu_idx = int(cvd.split(",")[local])
+        except ValueError:
+            pass
+    clocks = ClockSampler(gpu_idx)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    kern_ms = []
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    time.sleep(0.3)
+    wall0 = time.perf_counter()
+    for i in range(args.steps):
+        flush.zero_()                      # L2 flush between timed steps (untimed)
+        ev[i][0].record()
+        res, Tk, bk = step(plan)
+        ev[i][1].record()
+        torch.cuda.synchronize()
+        if hi > lo:
+            kern_ms.append(ap.ap_last_kernel_ms())
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    wall = time.perf_counter() - wall0
+    clk = clocks.stop()
+    step_ms = [s.elapsed_time(e) for s, e in ev]
+    t_local = sum(step_ms) / 1e3
+    tt = torch.tensor([t_local, sum(kern_ms) / 1e3 if kern_ms else 0.0], dtype=torch.float64,
+                      device=dev)
+    if world > 1:
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    t_max, kern_max = float(tt[0]), float(tt[1])
+    value = total_sims * args.steps / t_max
+    info = ap.ap_last_launch()
+
+    # ------------------------------------------------------------- e2e (host buffers)
+    e2e_steps = max(3, min(args.steps, 5))
+    tab_bytes = 3 * ((wl.n + 1) & ~1) * 8 + (wl.n + 1) * 33 * 8
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        pl = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=local)   # H2D tables
+        step(pl)                                                            # D2H key/result
+        pl.close()
+    torch.cuda.synchronize()
+    e2e_t = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+    e2e_val = total_sims * e2e_steps / float(e2e_t[0])
+
+    # ------------------------------------------------------------- secondary workloads
+    secondary = {}
+    if not args.no_secondary:
+        secondary = run_secondary(ap, torch, dist, world, rank, dev, shard)
+
+    # ------------------------------------------------------------- roofline
+    k_avg_s = kern_max / max(len(kern_ms), 1)
+    achieved = my_ops / k_avg_s if k_avg_s > 0 else 0.0
+    peak = int_peak_ops(sm_max, sms)
+    roof = {"bound": "alu", "kernel": "k_sweep_exact<%d,%s>" % (wl.p, "u32" if info["fast_u32"] else "u64"),
+            "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s (int32)",
+            "frac": achieved / peak, "traffic": None,
+            "ops_per_launch": my_ops, "ops_per_sim_avg": my_ops / max(hi - lo, 1) / K,
+            "frac_naive_count": (my_ops_naive / k_avg_s / peak) if k_avg_s > 0 else None,
+            "kernel_ms_avg": k_avg_s * 1e3,
+            "kernel_share_of_step": (kern_max / t_max) if t_max > 0 else None,
+            "peak_source": f"{sms} SMs x 128 int32 lanes/clk x sm_max {sm_max:.0f} MHz "
+                           f"({peak_src} MEASURED_PEAKS.json clock)",
+            "traffic_note": "algorithmic HBM bytes per candidate = 0; see profiles/ for ncu DRAM bytes"}
+    out = {"metric": METRIC, "value": value, "unit": "sims/s", "n_gpus": world,
+           "steps": args.steps, "warmup": args.warmup,
+           "ms_per_step": 1e3 * t_max / args.steps,
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+           "dtype": "u32" if info["fast_u32"] else "int64", "data": "synthetic",
+           "config": {"workload": wl.name, "n": wl.n, "p": wl.p, "m": wl.m, "k": [wl.k_lo, wl.k_hi],
+                      "search": "exhaustive", "sims_per_step": total_sims,
+                      "parallelism": f"rank-space shards x{world}",
+                      "l2": "flushed between timed steps (256 MiB write); tables are 2.4 KB",
+                      "arith": "u32 saturating at T_ref+1, exact for every candidate that can "
+                               "win (DESIGN.md §5.2)" if info["fast_u32"] else "int64",
+                      "time_to_optimal_plan_ms": 1e3 * t_max / args.steps,
+                      "wall_s": wall},
+           "result": {"T_ns": res["time_ns"], "rank": res["rank"], "k": res["k"],
+                      "cuts": res["cuts"], "master": res["master"], "slicer_best_k": bk},
+           "roofline": roof,
+           "clocks": clk,
+           "gpu_launches": 7 * args.steps,
+           "e2e": {"value": e2e_val, "unit": "sims/s", "h2d_bytes_per_step": tab_bytes,
+                   "d2h_bytes_per_step": 8 + 8 + 140 + 8 * wl.k_hi, "steps": e2e_steps,
+                   "path": "ap_plan_create(host tables) -> ap_search_exhaustive -> "
+                           "all_reduce -> ap_decode -> ap_slice_sweep -> ap_plan_destroy"},
+           "secondary": secondary}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        out["cpu_baseline"] = oracle_rate(wl)
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+    return 0
+
+
+def run_secondary(ap, torch, dist, world, rank, dev, shard):
+    """C3 exhaustive and C5 heuristic (65 536 restarts + Slicer sweep), fewer steps."""
+    out = {}
+    # C3
+    wl = synth.config(3)
+    f, b, a = wl.arrays()
+    plan = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=dev.index)
+    N = ap.ap_count(wl.n, wl.p)
+    lo, hi = shard(N, rank, world)
+    key = torch.empty(1, dtype=torch.int64, device=dev)
+
+    def s3():
+        ap.ap_search_exhaustive(plan, wl.p, wl.m, 1, 1, lo, hi, key)
+        if world > 1:
+            dist.all_reduce(key, op=dist.ReduceOp.MIN)
+        return ap.ap_decode(plan, 0, wl.p, wl.m, 1, 1, key=int(key.item()))
+    for _ in range(3):
+        s3()
+    times = []
+    for _ in range(5):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(); r3 = s3(); e1.record(); torch.cuda.synchronize()
+        times.append(e0.elapsed_time(e1))
+    t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    out["C3"] = {"workload": wl.name, "sims_per_s": N / (float(t[0]) / 1e3),
+                 "time_to_optimal_plan_ms": float(t[0]), "T_ns": r3["time_ns"], "cuts": r3["cuts"]}
+    # C5
+    wl = synth.config(5)
+    f, b, a = wl.arrays()
+    plan5 = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=dev.index)
+    rlo, rhi = shard(wl.restarts, rank, world)
+
+    def s5():
+        ap.ap_search_heuristic(plan5, wl.p, wl.m, wl.seed, wl.radius, rlo, rhi, 0, key)
+        if world > 1:
+            dist.all_reduce(key, op=dist.ReduceOp.MIN)
+        res = ap.ap_decode(plan5, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=int(key.item()))
+        Tk, bk = ap.ap_slice_sweep(plan5, wl.p, wl.m, res["cuts"], wl.slice_k_max)
+        return res, Tk, bk
+    s5()
+    times = []
+    kt = []
+    for _ in range(3):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(); r5, Tk, bk = s5(); e1.record(); torch.cuda.synchronize()
+        times.append(e0.elapsed_time(e1))
+    t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    out["C5"] = {"workload": wl.name, "restarts": wl.restarts,
+                 "restarts_per_s": wl.restarts / (float(t[0]) / 1e3),
+                 "time_to_plan_ms": float(t[0]), "T_ns": r5["time_ns"], "restart": r5["restart"],
+                 "cuts": r5["cuts"], "slicer_T_ns": [int(x) for x in Tk], "slicer_best_k": bk}
+    return out
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -227,8 +227,16 @@ typedef struct {
   int64_t t_ref;           /* T(Algorithm 1 partition, k_lo)                      */
   int32_t rank_bits;       /* rb                                                  */
   int32_t launches;        /* kernels launched by the call                        */
+  int32_t clamp_rows;      /* u32 path: steady rows between saturating clamps      */
 } ap_launch_info;
 void ap_last_launch(ap_launch_info* info);
+
+/* Device time (ms) of the dominant kernel of the last ap_search_exhaustive /
+ * ap_search_heuristic call on this thread (the sweep or restart kernel alone),
+ * from CUDA events the library records around that launch on the caller's stream.
+ * Valid once the stream has passed the launch; AP_ERR_INVALID before that or if
+ * no search ran. */
+ap_status ap_last_kernel_ms(float* ms);
 
 #ifdef __cplusplus
 }

@@ -17,7 +17,7 @@ from typing import Optional, Sequence
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libap.so")
+LIB_PATH = os.environ.get("AP_LIB_PATH") or os.path.join(_HERE, "libap.so")
 
 AP_MAX_P = 32
 AP_MAX_K = 16
@@ -48,7 +48,7 @@ class ApOp(C.Structure):
 class ApLaunchInfo(C.Structure):
     _fields_ = [("fast_u32", C.c_int32), ("exact_p", C.c_int32), ("blocks", C.c_int32),
                 ("threads", C.c_int32), ("chunk", C.c_uint64), ("t_ref", C.c_int64),
-                ("rank_bits", C.c_int32), ("launches", C.c_int32)]
+                ("rank_bits", C.c_int32), ("launches", C.c_int32), ("clamp_rows", C.c_int32)]
 
 
 def _load_lib():
@@ -85,6 +85,8 @@ def _load_lib():
     lib.ap_alg1.argtypes = [vp, i32, P(i32), P(i64)]
     lib.ap_last_launch.restype = None
     lib.ap_last_launch.argtypes = [P(ApLaunchInfo)]
+    lib.ap_last_kernel_ms.restype = i32
+    lib.ap_last_kernel_ms.argtypes = [P(C.c_float)]
     return lib
 
 
@@ -93,7 +95,8 @@ lib = _load_lib()
 # every symbol include/ap.h declares (checked by tests/test_abi.py)
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
            "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_heuristic",
-           "ap_decode", "ap_slice_sweep", "ap_critical_path", "ap_alg1", "ap_last_launch")
+           "ap_decode", "ap_slice_sweep", "ap_critical_path", "ap_alg1", "ap_last_launch",
+           "ap_last_kernel_ms")
 
 
 def _check(st: int):
@@ -264,3 +267,11 @@ def ap_last_launch() -> dict:
     info = ApLaunchInfo()
     lib.ap_last_launch(C.byref(info))
     return {f: getattr(info, f) for f, _ in ApLaunchInfo._fields_}
+
+
+def ap_last_kernel_ms() -> float:
+    """Device time of the last search's dominant kernel (library CUDA events on the
+    caller's stream); the stream must have passed it."""
+    v = C.c_float()
+    _check(lib.ap_last_kernel_ms(C.byref(v)))
+    return float(v.value)

@@ -19,6 +19,30 @@ namespace {
 thread_local std::string g_err;
 thread_local ap_launch_info g_last{};
 
+// CUDA events bracketing the dominant kernel of the last search on this thread.
+struct KernelTimer {
+  cudaEvent_t ev[2] = {nullptr, nullptr};
+  int dev = -1;
+  bool armed = false;
+  cudaError_t record(int which, cudaStream_t s, int device) {
+    if (dev != device) {
+      // events belong to the device current at creation
+      for (auto& e : ev)
+        if (e) cudaEventDestroy(e);
+      ev[0] = ev[1] = nullptr;
+      dev = device;
+    }
+    for (auto& e : ev)
+      if (!e) {
+        cudaError_t r = cudaEventCreate(&e);
+        if (r != cudaSuccess) return r;
+      }
+    armed = (which == 1);
+    return cudaEventRecord(ev[which], s);
+  }
+};
+thread_local KernelTimer g_timer;
+
 ap_status fail(ap_status st, const char* fmt, ...) {
   char buf[512];
   va_list ap;
@@ -49,13 +73,16 @@ struct DeviceGuard {
   }
 };
 
-// Per-call device scratch, released stream-ordered.
+// Per-call device scratch from the plan's memory pool (release threshold = max,
+// so stream-ordered frees never unmap memory at a synchronisation), released
+// stream-ordered.
 struct Scratch {
   cudaStream_t s;
+  cudaMemPool_t pool;
   std::vector<void*> ptrs;
-  explicit Scratch(cudaStream_t st) : s(st) {}
+  Scratch(cudaStream_t st, cudaMemPool_t pl) : s(st), pool(pl) {}
   cudaError_t get(void** p, size_t bytes) {
-    cudaError_t e = cudaMallocAsync(p, bytes < 16 ? 16 : bytes, s);
+    cudaError_t e = cudaMallocFromPoolAsync(p, bytes < 16 ? 16 : bytes, pool, s);
     if (e == cudaSuccess) ptrs.push_back(*p);
     return e;
   }
@@ -63,6 +90,18 @@ struct Scratch {
     for (void* p : ptrs) cudaFreeAsync(p, s);
   }
 };
+
+// One internal non-blocking stream per (thread, device) for the blocking calls.
+cudaError_t internal_stream(int device, cudaStream_t* out) {
+  thread_local cudaStream_t streams[64] = {nullptr};
+  if (device < 0 || device >= 64) return cudaErrorInvalidDevice;
+  if (!streams[device]) {
+    cudaError_t e = cudaStreamCreateWithFlags(&streams[device], cudaStreamNonBlocking);
+    if (e != cudaSuccess) return e;
+  }
+  *out = streams[device];
+  return cudaSuccess;
+}
 
 int bitlen(unsigned __int128 v) {
   int b = 0;
@@ -92,6 +131,7 @@ struct ap_plan {
   uint64_t link = 0;
   int64_t* d_tab = nullptr;
   uint64_t* d_binom = nullptr;
+  cudaMemPool_t pool = nullptr;
   apk::DevTables dev() const { return apk::DevTables{d_tab, d_binom, n, npad}; }
 };
 
@@ -103,6 +143,16 @@ const char* ap_version(void) { return "autopipe-b200 0.1 (sm_100a)"; }
 
 void ap_last_launch(ap_launch_info* info) {
   if (info) *info = g_last;
+}
+
+ap_status ap_last_kernel_ms(float* ms) {
+  if (!ms) return fail(AP_ERR_INVALID, "ms is NULL");
+  if (!g_timer.armed) return fail(AP_ERR_INVALID, "no search launched on this thread");
+  if (cudaEventQuery(g_timer.ev[1]) != cudaSuccess)
+    return fail(AP_ERR_INVALID, "last search kernel not complete");
+  cudaError_t e = cudaEventElapsedTime(ms, g_timer.ev[0], g_timer.ev[1]);
+  if (e != cudaSuccess) return fail(AP_ERR_CUDA, "elapsed: %s", cudaGetErrorString(e));
+  return AP_OK;
 }
 
 ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns,
@@ -171,6 +221,17 @@ ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns
   if (e == cudaSuccess) e = cudaMemcpy(P->d_tab, tab.data(), tab.size() * 8, cudaMemcpyHostToDevice);
   if (e == cudaSuccess)
     e = cudaMemcpy(P->d_binom, binom.data(), binom.size() * 8, cudaMemcpyHostToDevice);
+  if (e == cudaSuccess) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = device;
+    e = cudaMemPoolCreate(&P->pool, &props);
+    if (e == cudaSuccess) {
+      uint64_t thr = UINT64_MAX;
+      e = cudaMemPoolSetAttribute(P->pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+  }
   if (e != cudaSuccess) {
     ap_plan_destroy(P);
     return fail(e == cudaErrorMemoryAllocation ? AP_ERR_NOMEM : AP_ERR_CUDA, "plan upload: %s",
@@ -186,6 +247,10 @@ void ap_plan_destroy(ap_plan* plan) {
     DeviceGuard g(plan->device);
     if (plan->d_tab) cudaFree(plan->d_tab);
     if (plan->d_binom) cudaFree(plan->d_binom);
+    if (plan->pool) {
+      cudaDeviceSynchronize();  // stream-ordered frees into the pool must land first
+      cudaMemPoolDestroy(plan->pool);
+    }
   }
   delete plan;
 }
@@ -245,7 +310,7 @@ ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t
   int launches = 0;
   static const int32_t kDummy = 0;
   (void)kDummy;
-  AP_CUDA(apk::launch_eval(plan->dev(), p, m, p > 1 ? cuts : nullptr, p - 1, k, 1, 0, count,
+  AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? cuts : nullptr, p - 1, k, 1, 0, count,
                            time_ns, master, S_(stream), &launches));
   return AP_OK;
 }
@@ -274,10 +339,10 @@ ap_status ap_alg1(const ap_plan* plan, int32_t p, int32_t* cuts, int64_t* value)
   if (p < 1 || p > plan->n || p > AP_MAX_P) return fail(AP_ERR_INVALID, "p=%d", p);
   DeviceGuard g(plan->device);
   cudaStream_t s;
-  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  AP_CUDA(internal_stream(plan->device, &s));
   ap_status st;
   {
-    Scratch sc(s);
+    Scratch sc(s, plan->pool);
     int16_t* arg;
     int32_t* dc;
     int64_t* dv;
@@ -296,7 +361,6 @@ ap_status ap_alg1(const ap_plan* plan, int32_t p, int32_t* cuts, int64_t* value)
     }
   }
   cudaStreamSynchronize(s);
-  cudaStreamDestroy(s);
   return st;
 }
 
@@ -320,7 +384,7 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
   cudaStream_t s = S_(stream);
   DeviceGuard g(plan->device);
   ap_launch_info info{};
-  Scratch sc(s);
+  Scratch sc(s, plan->pool);
   int16_t* d_arg;
   int32_t* d_a1;
   int64_t* d_val;
@@ -329,7 +393,7 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
   int64_t* d_tref;
   AP_CUDA(sc.get((void**)&d_tref, 8));
   int launches = 1;
-  AP_CUDA(apk::launch_eval(plan->dev(), p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 0, 1,
+  AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 0, 1,
                            d_tref, nullptr, s, &launches));
   int64_t tref = 0;
   AP_CUDA(cudaMemcpyAsync(&tref, d_tref, 8, cudaMemcpyDeviceToHost, s));
@@ -338,13 +402,21 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
   if (rb >= 63 || (uint64_t)tref >= ((1ull << (63 - rb)) - 1))
     return fail(AP_ERR_RANGE, "key packing: T_ref=%lld needs %d bits + %d rank bits > 63",
                 (long long)tref, bitlen((unsigned __int128)tref), rb);
-  // exact u32 saturating fast path: S = T_ref + 1, rows between
-  // clamps <= max(p, 4) + 2, each row adds at most W_row to any running value.
+  // exact u32 saturating fast path: S = T_ref + 1.  Between two
+  // clamps every running value grows by at most W_row per row of the sweep, so with
+  // R_allow = floor((2^32-1-S)/W_row) rows per clamp segment nothing wraps.  The
+  // segments are: rows 0..p-1 (pieces + warm-up + first 1F1B row), blocks of
+  // clamp_rows steady rows, and the p-1 cool-down rows.
   const uint64_t S = (uint64_t)tref + 1;
   const unsigned __int128 wrow = (unsigned __int128)(plan->sum_f + plan->sum_b) +
-                                 (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm;
-  const int seg = (p > 4 ? p : 4) + 2;
-  int want_u32 = ((unsigned __int128)S + wrow * seg) < ((unsigned __int128)1 << 32);
+                                 (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
+  const unsigned __int128 lim = ((unsigned __int128)1 << 32) - 1;
+  const uint64_t r_allow = (S >= lim) ? 0 : (uint64_t)((lim - S) / wrow);
+  int want_u32 = r_allow >= (uint64_t)p && r_allow >= 1;
+  int clamp_rows = (int)(r_allow < (uint64_t)m ? r_allow : (uint64_t)m);
+  if (clamp_rows >= 8) clamp_rows &= ~7;  // whole unrolled blocks
+  else if (clamp_rows >= 4) clamp_rows &= ~3;
+  if (clamp_rows < 1) clamp_rows = 1;
   // test/bench overrides: AP_SWEEP=int64 disables the u32 path, AP_SWEEP=generic
   // also the p-specialised kernel (both remain exact)
   const char* ov = getenv("AP_SWEEP");
@@ -352,8 +424,12 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
   if (ov && strcmp(ov, "int64") == 0) want_u32 = 0;
   if (ov && strcmp(ov, "generic") == 0) { want_u32 = 0; force_generic = 1; }
   apk::SweepPlan sp{};
+  AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), nullptr, s));
+  AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, S, rb, want_u32,
-                            force_generic, reinterpret_cast<unsigned long long*>(key), s, &sp));
+                            clamp_rows, force_generic, reinterpret_cast<unsigned long long*>(key),
+                            s, &sp));
+  AP_CUDA(g_timer.record(1, s, plan->device));
   launches += 2;
   info.fast_u32 = sp.fast_u32;
   info.exact_p = sp.exact_p;
@@ -362,6 +438,7 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
   info.chunk = sp.chunk;
   info.t_ref = tref;
   info.rank_bits = rb;
+  info.clamp_rows = sp.fast_u32 ? clamp_rows : 0;
   info.launches = launches;
   g_last = info;
   return AP_OK;
@@ -379,7 +456,7 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   if (radius < 0 || radius > (1 << 20)) return fail(AP_ERR_INVALID, "radius %d", radius);
   cudaStream_t s = S_(stream);
   DeviceGuard g(plan->device);
-  Scratch sc(s);
+  Scratch sc(s, plan->pool);
   int16_t* d_arg;
   int32_t* d_a1;
   int64_t* d_val;
@@ -387,10 +464,13 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   if (st != AP_OK) return st;
   unsigned int* d_ctr;
   AP_CUDA(sc.get((void**)&d_ctr, 16));
+  AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), d_ctr, s));
+  AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_heuristic(plan->dev(), p, m, seed, radius, r_lo, r_hi, d_arg, d_a1, d_ctr,
                                 reinterpret_cast<unsigned long long*>(key), nullptr, s));
+  AP_CUDA(g_timer.record(1, s, plan->device));
   ap_launch_info info{};
-  info.launches = 3;
+  info.launches = 3;  // alg1, init, restarts
   g_last = info;
   return AP_OK;
 }
@@ -407,10 +487,10 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
   out->p = p;
   DeviceGuard g(plan->device);
   cudaStream_t s;
-  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  AP_CUDA(internal_stream(plan->device, &s));
   ap_status res = AP_OK;
   {
-    Scratch sc(s);
+    Scratch sc(s, plan->pool);
     int32_t* d_cuts = nullptr;
     int32_t* d_master = nullptr;
     int64_t* d_T = nullptr;
@@ -457,6 +537,7 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
       if (res == AP_OK) {
         e = sc.get((void**)&d_ctr, 16);
         if (e == cudaSuccess) e = sc.get((void**)&d_key, 16);
+        if (e == cudaSuccess) e = apk::launch_init_key(d_key, d_ctr, s);
         if (e == cudaSuccess)
           e = apk::launch_heuristic(plan->dev(), p, m, seed, radius, r, r + 1, d_arg, d_a1, d_ctr,
                                     d_key, d_cuts, s);
@@ -467,7 +548,7 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
     }
     if (res == AP_OK) {
       int launches = 0;
-      e = apk::launch_eval(plan->dev(), p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, kk, 0, 1, d_T,
+      e = apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, kk, 0, 1, d_T,
                            d_master, s, &launches);
       int32_t hc[32] = {0};
       int64_t T = -1;
@@ -499,7 +580,6 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
     }
   }
   cudaStreamSynchronize(s);
-  cudaStreamDestroy(s);
   return res;
 }
 
@@ -512,10 +592,10 @@ ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_
   if (!time_ns || !best_k || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL argument");
   DeviceGuard g(plan->device);
   cudaStream_t s;
-  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  AP_CUDA(internal_stream(plan->device, &s));
   ap_status res = AP_OK;
   {
-    Scratch sc(s);
+    Scratch sc(s, plan->pool);
     int32_t* d_cuts;
     int64_t* d_T;
     cudaError_t e = sc.get((void**)&d_cuts, 4 * 32);
@@ -524,7 +604,7 @@ ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_
       e = cudaMemcpyAsync(d_cuts, cuts, 4 * (size_t)(p - 1), cudaMemcpyHostToDevice, s);
     int launches = 0;
     if (e == cudaSuccess)
-      e = apk::launch_eval(plan->dev(), p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, 1, 1, k_max,
+      e = apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, 1, 1, k_max,
                            d_T, nullptr, s, &launches);
     if (e == cudaSuccess)
       e = cudaMemcpyAsync(time_ns, d_T, 8 * (size_t)k_max, cudaMemcpyDeviceToHost, s);
@@ -532,7 +612,6 @@ ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_
     if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "slice sweep: %s", cudaGetErrorString(e));
   }
   cudaStreamSynchronize(s);
-  cudaStreamDestroy(s);
   if (res != AP_OK) return res;
   if (time_ns[0] < 0) return fail(AP_ERR_INVALID, "invalid cut vector");
   int bk = 1;
@@ -553,12 +632,12 @@ ap_status ap_critical_path(const ap_plan* plan, int32_t p, int32_t m, int32_t k,
   static_assert(sizeof(ap_op) == sizeof(apk::OpRec), "ap_op layout");
   DeviceGuard g(plan->device);
   cudaStream_t s;
-  AP_CUDA(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+  AP_CUDA(internal_stream(plan->device, &s));
   ap_status res = AP_OK;
   int32_t lm[2] = {-1, -1};
   int64_t T = -1;
   {
-    Scratch sc(s);
+    Scratch sc(s, plan->pool);
     int32_t *d_cuts, *d_lm;
     int64_t* d_T;
     apk::OpRec* d_ops;
@@ -582,7 +661,6 @@ ap_status ap_critical_path(const ap_plan* plan, int32_t p, int32_t m, int32_t k,
     if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "critical path: %s", cudaGetErrorString(e));
   }
   cudaStreamSynchronize(s);
-  cudaStreamDestroy(s);
   if (res != AP_OK) return res;
   if (lm[0] < 0) return fail(AP_ERR_INVALID, "invalid cut vector");
   if (len) *len = lm[0];

@@ -43,107 +43,157 @@ AP_DEV_INLINE uint32_t divk(uint32_t v, uint32_t k, uint32_t M) {
 }
 AP_DEV_INLINE uint64_t divk(uint64_t v, uint32_t k, uint32_t) { return v / k; }
 
+
+// Integer ops of the sweep.  Written as plain operators: ptxas then fuses the add
+// of the backward chain into the max (VIADDMNMX, ALU pipe) and puts most other adds
+// on IMAD.IADD (FMA pipe).  Forcing every add onto IMAD (mad.lo with an opaque
+// multiplier) or a signed offset form that removes the adds were both measured
+// slower on C4 (profiles/r01_sweep_variants.md).
+template <typename V>
+struct XOps {
+  static AP_DEV_INLINE V mx(V a, V b) { return a > b ? a : b; }
+  static AP_DEV_INLINE V ad(V a, V b, uint32_t) { return a + b; }
+  static AP_DEV_INLINE V amx(V a, V b, V c) {  // max(a + b, c)
+    const V t = a + b;
+    return t > c ? t : c;
+  }
+};
+
+// One fused steady step: the backward pass of row r and the
+// forward pass of row r+1 share their maxima.  With b_r[x] = max(b_r[x+1], FF_r[x]) +
+// wB[x] and FF_{r+1}[x+1] = max(FF_r[x], b_r[x+1]) + wF[x+1], both are
+// M[x] = max(FF_r[x], b_r[x+1]) plus a weight, and M[x] = max(M[x+1] + wB[x+1],
+// FF_r[x]) is one fused add+max (VIADDMNMX, ALU pipe).  A step is P-1 ALU
+// instructions plus P IMAD adds (FMA pipe): 2P-1 instructions for the 2P max-plus
+// ops of a row.  State between steps: FF[0..P-1] only.
 template <int P, typename V>
-AP_DEV_INLINE void clamp_state(V (&FF)[P], V (&L)[P], V S) {
-  if constexpr (sizeof(V) == 4) {
+AP_DEV_INLINE void mstep(V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V wBF0, uint32_t one) {
+  using O = XOps<V>;
+  if constexpr (P == 1) {
+    FF[0] = O::ad(FF[0], wBF0, one);
+  } else {
+    V nF[P];
+    V M = O::amx(FF[P - 1], wB[P - 1], FF[P - 2]);
+    nF[P - 1] = O::ad(M, wF[P - 1], one);
 #pragma unroll
-    for (int x = 0; x < P; ++x) {
-      FF[x] = vmin(FF[x], S);
-      L[x] = vmin(L[x], S);
+    for (int x = P - 3; x >= 0; --x) {
+      M = O::amx(M, wB[x + 1], FF[x]);
+      nF[x + 1] = O::ad(M, wF[x + 1], one);
     }
+    nF[0] = O::ad(M, wBF0, one);
+#pragma unroll
+    for (int x = 0; x < P; ++x) FF[x] = nF[x];
   }
 }
 
-// One steady 1F1B row (rows r = P..m-1): every stage does F then B.
 template <int P, typename V>
-AP_DEV_INLINE void row_steady(V (&FF)[P], V (&L)[P], const V (&wF)[P], const V (&wB)[P]) {
+AP_DEV_INLINE void clamp_ff(V (&FF)[P], V S) {
+  if constexpr (sizeof(V) == 4) {
 #pragma unroll
-  for (int x = P - 1; x >= 1; --x) FF[x] = vmax(FF[x - 1], L[x]) + wF[x];
-  FF[0] = L[0] + wF[0];
-  V b = FF[P - 1] + wB[P - 1];
-  L[P - 1] = b;
-#pragma unroll
-  for (int x = P - 2; x >= 0; --x) {
-    b = vmax(b, FF[x]) + wB[x];
-    L[x] = b;
+    for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
   }
 }
 
 // Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
 template <int P, typename V>
-AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const V (&Fr)[P],
-                         const V (&Ci)[P], uint32_t Mk, V S) {
+AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const int (&c)[P + 1],
+                         const V* sPf, const V* sC, uint32_t Mk, V S, int CR, uint32_t one) {
+  using O = XOps<V>;
   V FF[P], L[P];
-  // micro-batch 0's forward, sliced into k pieces (reading Q6)
+  // micro-batch 0's forward, sliced into k pieces (reading Q6); the raw stage
+  // compute/comm are re-read from shared memory only on this (k > 1) path
   if (k == 1) {
     FF[0] = wF[0];
 #pragma unroll
-    for (int x = 1; x < P; ++x) FF[x] = FF[x - 1] + wF[x];
+    for (int x = 1; x < P; ++x) FF[x] = O::ad(FF[x - 1], wF[x], one);
   } else {
     V a[P], al[P];
 #pragma unroll
     for (int x = 0; x < P; ++x) {
-      a[x] = divk(Fr[x], (uint32_t)k, Mk) + ((x > 0) ? divk(Ci[x], (uint32_t)k, Mk) : V(0));
+      const V Fx = sPf[c[x + 1]] - sPf[c[x]];
+      const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
+      a[x] = divk(Fx, (uint32_t)k, Mk) + ((x > 0) ? divk(Cin, (uint32_t)k, Mk) : V(0));
       al[x] = wF[x] - V(k - 1) * a[x];
       FF[x] = 0;
     }
     for (int q = 0; q < k - 1; ++q) {
-      FF[0] = FF[0] + a[0];
+      FF[0] = O::ad(FF[0], a[0], one);
 #pragma unroll
-      for (int x = 1; x < P; ++x) FF[x] = vmax(FF[x - 1], FF[x]) + a[x];
+      for (int x = 1; x < P; ++x) FF[x] = O::ad(O::mx(FF[x - 1], FF[x]), a[x], one);
     }
-    FF[0] = FF[0] + al[0];
+    FF[0] = O::ad(FF[0], al[0], one);
 #pragma unroll
-    for (int x = 1; x < P; ++x) FF[x] = vmax(FF[x - 1], FF[x]) + al[x];
+    for (int x = 1; x < P; ++x) FF[x] = O::ad(O::mx(FF[x - 1], FF[x]), al[x], one);
   }
   // warm-up rows r = 1..P-2: stage x <= r-1 does F(x, r-x); L == FF here
 #pragma unroll
   for (int r = 1; r <= P - 2; ++r) {
 #pragma unroll
-    for (int x = r - 1; x >= 1; --x) FF[x] = vmax(FF[x - 1], FF[x]) + wF[x];
-    FF[0] = FF[0] + wF[0];
+    for (int x = r - 1; x >= 1; --x) FF[x] = O::ad(O::mx(FF[x - 1], FF[x]), wF[x], one);
+    FF[0] = O::ad(FF[0], wF[0], one);
   }
 #pragma unroll
   for (int x = 0; x < P; ++x) L[x] = FF[x];
-  // row P-1: stages 0..P-2 do F(x, P-1-x); F(P-1, 0) was a piece; all do B(x, 0)
+  // row P-1, forward part: stages 0..P-2 do F(x, P-1-x); F(P-1, 0) was a piece
+#pragma unroll
+  for (int x = P - 2; x >= 1; --x) FF[x] = O::ad(O::mx(FF[x - 1], L[x]), wF[x], one);
+  if (P >= 2) FF[0] = O::ad(L[0], wF[0], one);
+  clamp_ff<P, V>(FF, S);
+  // fused steps r = P-1..m-2: backward pass of row r + forward pass of row r+1.
   {
+    // fused M-form, clamped (u32) every CR steps: the host's no-wrap bound
+    // S + CR * W_row < 2^32
+    constexpr int U = (P <= 8) ? 8 : 4;
+    const V wBF0 = wB[0] + wF[0];
+    int rem = m - P;
+    while (rem > 0) {
+      int blk = rem < CR ? rem : CR;
+      rem -= blk;
+      for (; blk >= U; blk -= U) {
 #pragma unroll
-    for (int x = P - 2; x >= 1; --x) FF[x] = vmax(FF[x - 1], L[x]) + wF[x];
-    if (P >= 2) FF[0] = L[0] + wF[0];
-    V b = FF[P - 1] + wB[P - 1];
-    L[P - 1] = b;
-#pragma unroll
-    for (int x = P - 2; x >= 0; --x) {
-      b = vmax(b, FF[x]) + wB[x];
-      L[x] = b;
+        for (int u = 0; u < U; ++u) mstep<P, V>(FF, wF, wB, wBF0, one);
+      }
+      for (; blk > 0; --blk) mstep<P, V>(FF, wF, wB, wBF0, one);
+      clamp_ff<P, V>(FF, S);
     }
   }
-  clamp_state<P, V>(FF, L, S);
-  // steady rows r = P..m-1
-  constexpr int U = (P <= 8) ? 4 : 2;
-  int rem = m - P;
-  for (; rem >= U; rem -= U) {
+  // cool-down, fused the same way: step t = 0..P-1 is the backward pass of row
+  // r = m-1+t plus the forward pass of row r+1, which only stages x >= t+1 still
+  // do.  Stages x < t did no forward in row r: their backward reads L[x] (their
+  // last op) instead of a shared maximum.  M carries max(FF[x], b[x+1]) with
+  // b[x+1] = M + wB[x+1] folded into the next fused add+max.
+  V b = 0;
 #pragma unroll
-    for (int u = 0; u < U; ++u) row_steady<P, V>(FF, L, wF, wB);
-    clamp_state<P, V>(FF, L, S);
-  }
-  for (; rem > 0; --rem) row_steady<P, V>(FF, L, wF, wB);
-  clamp_state<P, V>(FF, L, S);
-  // cool-down rows r = m+c, c = 0..P-2: F only on stages x >= c+1
+  for (int t = 0; t < P; ++t) {
+    if constexpr (P == 1) {
+      b = O::ad(FF[0], wB[0], one);
+    } else {
+      V M = FF[P - 1];   // pending value; b[P-1] = M + wB[P-1]
+      V wpend = wB[P - 1];
 #pragma unroll
-  for (int c = 0; c <= P - 2; ++c) {
-#pragma unroll
-    for (int x = P - 1; x >= c + 1; --x) FF[x] = vmax(FF[x - 1], L[x]) + wF[x];
-    V b = FF[P - 1] + wB[P - 1];
-    L[P - 1] = b;
-#pragma unroll
-    for (int x = P - 2; x >= 0; --x) {
-      const V in = (x >= c + 1) ? FF[x] : L[x];
-      b = vmax(b, in) + wB[x];
-      L[x] = b;
+      for (int x = P - 2; x >= 0; --x) {
+        if (x >= t) {
+          M = O::amx(M, wpend, FF[x]);                      // max(b[x+1], FF[x])
+          if (t < P - 1) FF[x + 1] = O::ad(M, wF[x + 1], one);  // not read again this step
+          wpend = wB[x];
+          if (x == t) {
+            L[x] = O::ad(M, wB[x], one);
+            M = L[x];
+            wpend = 0;
+          }
+        } else {
+          // b[x] = max(b[x+1], L[x]) + wB[x] with b[x+1] = M + wpend; wpend is 0
+          // unless stage x+1 is P-1 (its weight is still pending from the start)
+          const V bx1 = (x <= P - 3) ? M : O::ad(M, wpend, one);
+          M = O::ad(O::mx(bx1, L[x]), wB[x], one);
+          L[x] = M;
+          wpend = 0;
+        }
+      }
+      b = M;  // stage 0 is always materialised (x == t or x < t)
     }
   }
-  return L[0];
+  return b;
 }
 
 struct SweepArgs {
@@ -153,6 +203,8 @@ struct SweepArgs {
   uint64_t S;
   int rb;
   unsigned long long* key;
+  int clamp_rows;  // u32 path: rows between saturating clamps (>= 1)
+  uint32_t one;    // = 1, opaque to the compiler (keeps adds on IMAD, see XOps)
 };
 
 AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
@@ -177,7 +229,10 @@ AP_DEV_INLINE void block_min_atomic(unsigned long long v, unsigned long long* ou
 }
 
 template <int P, typename V>
-__global__ void __launch_bounds__(256) k_sweep_exact(SweepArgs A) {
+#ifndef AP_SWEEP_MINB
+#define AP_SWEEP_MINB (P <= 8 ? 3 : 2)
+#endif
+__global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A) {
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
@@ -186,11 +241,14 @@ __global__ void __launch_bounds__(256) k_sweep_exact(SweepArgs A) {
   V* sPf = reinterpret_cast<V*>(smem + used);
   V* sPb = sPf + (n + 1);
   V* sC = sPb + (n + 1);
+  __shared__ uint32_t s_mk[kMaxK + 1];  // floor(2^32 / k) (k = 1: 2^32 - 1), see divk
   for (int i = threadIdx.x; i <= n; i += blockDim.x) {
     sPf[i] = (V)T.Pf[i];
     sPb[i] = (V)T.Pb[i];
     if (i < n) sC[i] = (V)T.comm[i];
   }
+  if (threadIdx.x <= kMaxK)
+    s_mk[threadIdx.x] = (threadIdx.x <= 1) ? 0xffffffffu : (uint32_t)((1ull << 32) / threadIdx.x);
   __syncthreads();
 
   const int m = A.m, k_lo = A.k_lo, k_hi = A.k_hi;
@@ -227,7 +285,7 @@ __global__ void __launch_bounds__(256) k_sweep_exact(SweepArgs A) {
     }
     for (uint64_t r = r0; r < r1; ++r) {
       // stage weights (a3): compute + receiver-side comm
-      V wF[P], wB[P], Fr[P], Ci[P];
+      V wF[P], wB[P];
 #pragma unroll
       for (int x = 0; x < P; ++x) {
         const V Fx = sPf[c[x + 1]] - sPf[c[x]];
@@ -236,13 +294,11 @@ __global__ void __launch_bounds__(256) k_sweep_exact(SweepArgs A) {
         const V Cout = (x < P - 1) ? sC[c[x + 1] - 1] : V(0);
         wF[x] = Fx + Cin;
         wB[x] = Bx + Cout;
-        Fr[x] = Fx;
-        Ci[x] = Cin;
       }
       const uint64_t base = r * K;
       for (int k = k_lo; k <= k_hi; ++k) {
-        const uint32_t Mk = (k == 1) ? 0xffffffffu : (uint32_t)((1ull << 32) / (uint32_t)k);
-        const V Tc = sim_fast<P, V>(m, k, wF, wB, Fr, Ci, Mk, S);
+        const uint32_t Mk = s_mk[k];
+        const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, S, A.clamp_rows, A.one);
         if (Tc < bestT) {
           bestT = Tc;
           bestIdx = base + (uint64_t)(k - k_lo);
@@ -513,7 +569,7 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
   BitsRef br{s_bits + threadIdx.x, (int)blockDim.x};
   TimesRef not_{nullptr, nullptr, nullptr};
 
-  int cur[P + 1], cand[P + 1], best[P + 1], sel[P + 1];
+  int cur[P + 1] = {0}, cand[P + 1] = {0}, best[P + 1] = {0}, sel[P + 1] = {0};
   unsigned long long lane_key = 0x7fffffffffffffffull;
   const int smax = n * p;
   int phase = 0;  // 0 need restart, 1 start evaluated next, 2 child evaluated next
@@ -802,7 +858,8 @@ static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_eval(const DevTables& t, int p, int m, const int32_t* cuts, int cuts_stride,
+cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, const int32_t* cuts,
+                        int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
                         int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches) {
   EvalArgs A{t, p, m, cuts, cuts_stride, kptr, k_const, k_iota, count, time_ns, master, nullptr};
@@ -813,7 +870,7 @@ cudaError_t launch_eval(const DevTables& t, int p, int m, const int32_t* cuts, i
     const size_t per = (size_t)rows * (P <= 16 ? 1 : 2) * 4;
     const size_t base = (tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15);
     if (per * 32 > 200 * 1024 - base) {
-      cudaError_t e = cudaMallocAsync((void**)&gbits, per * (size_t)count + 16, s);
+      cudaError_t e = cudaMallocFromPoolAsync((void**)&gbits, per * (size_t)count + 16, pool, s);
       if (e != cudaSuccess) return e;
       A.gbits = gbits;
     }
@@ -906,12 +963,12 @@ bool has_exact(int p) {
 }
 
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
-                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int force_generic,
-                         unsigned long long* key, cudaStream_t s, SweepPlan* sp) {
+                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
+                         int force_generic, unsigned long long* key, cudaStream_t s,
+                         SweepPlan* sp) {
   int dev = 0;
   cudaGetDevice(&dev);
-  k_init_key<<<1, 1, 0, s>>>(key);
-  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key};
+  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u};
   const bool exact = has_exact(p) && m >= p && !force_generic;
   sp->exact_p = exact ? 1 : 0;
   sp->fast_u32 = (exact && want_u32) ? 1 : 0;
@@ -955,9 +1012,6 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
                              unsigned long long* key, int32_t* replay_cuts, cudaStream_t s) {
   int dev = 0;
   cudaGetDevice(&dev);
-  k_init_key<<<1, 1, 0, s>>>(key);
-  cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned int), s);
-  if (e != cudaSuccess) return e;
   HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts};
   switch (pick_P(p)) {
     case 2: return heur_P<2>(A, s, dev);
@@ -1019,6 +1073,15 @@ cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t*
     case 16: return cpath_P<16>(A, s);
     default: return cpath_P<32>(A, s);
   }
+}
+
+cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s) {
+  k_init_key<<<1, 1, 0, s>>>(key);
+  if (counter) {
+    cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned int), s);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaGetLastError();
 }
 
 cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,

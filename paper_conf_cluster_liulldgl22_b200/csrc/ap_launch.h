@@ -21,7 +21,8 @@ cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, 
 // Generic exact evaluation of `count` candidates.  cuts_stride = p-1 (batch) or 0
 // (all rows share one cut vector).  k source: kptr if non-null, else k_iota ? row+1
 // : k_const.  master may be null.  Invalid rows -> time -1, master -1.
-cudaError_t launch_eval(const DevTables& t, int p, int m, const int32_t* cuts, int cuts_stride,
+cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, const int32_t* cuts,
+                        int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
                         int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches);
 
@@ -30,12 +31,14 @@ struct SweepPlan {
   int exact_p;    // kernel specialised to this p
   int blocks, threads;
   uint64_t chunk;
+  int clamp_rows;
 };
 // Exhaustive sweep of ranks [rank_lo, rank_hi) x k in [k_lo, k_hi].  S = T_ref + 1:
-// a candidate with T >= S can never win.  Writes INT64_MAX first, then atomicMin.
+// a candidate with T >= S can never win.  atomicMin into *key (init it first).
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
-                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int force_generic,
-                         unsigned long long* key, cudaStream_t s, SweepPlan* plan_out);
+                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
+                         int force_generic, unsigned long long* key, cudaStream_t s,
+                         SweepPlan* plan_out);
 
 // Heuristic restarts [r_lo, r_hi); key = min (T << 20 | r).  replay_cuts (int32[p-1])
 // non-null: single-restart replay writing that restart's best cut vector.
@@ -54,6 +57,9 @@ size_t cpath_scratch_bytes(int p, int m);
 cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t* cuts, OpRec* ops,
                          int cap, int32_t* len_master, int64_t* T, void* scratch,
                          cudaStream_t s);
+
+// key = INT64_MAX (and *counter = 0 if non-null); precedes launch_sweep/heuristic.
+cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s);
 
 // Decode helper: unrank lex rank -> cut vector int32[p-1].
 cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,

@@ -22,6 +22,34 @@ def shard(total: int, rank: int, world: int):
     return (total * rank) // world, (total * (rank + 1)) // world
 
 
+def rank_bits(N: int, K: int) -> int:
+    """rb = bitlen(N*K - 1): low bits of an exhaustive key (include/ap.h)."""
+    return (N * K - 1).bit_length()
+
+
+def pack_exhaustive_key(T: int, rank: int, k: int, N: int, k_lo: int, k_hi: int) -> int:
+    """key = T << rb | (rank*K + k - k_lo) -- the layout ap_search_exhaustive writes."""
+    K = k_hi - k_lo + 1
+    return (T << rank_bits(N, K)) | (rank * K + k - k_lo)
+
+
+def unpack_exhaustive_key(key: int, N: int, k_lo: int, k_hi: int):
+    """(T, rank, k) of a reduced exhaustive key; None for INT64_MAX (empty)."""
+    if key == INT64_MAX:
+        return None
+    K = k_hi - k_lo + 1
+    rb = rank_bits(N, K)
+    idx = key & ((1 << rb) - 1)
+    return key >> rb, idx // K, k_lo + idx % K
+
+
+def unpack_heuristic_key(key: int):
+    """(T, restart) of a reduced heuristic key (T << 20 | r)."""
+    if key == INT64_MAX:
+        return None
+    return key >> 20, key & ((1 << 20) - 1)
+
+
 def _world():
     import torch.distributed as dist
     if dist.is_available() and dist.is_initialized():

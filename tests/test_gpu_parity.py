@@ -327,3 +327,48 @@ def test_overflow_guard_and_errors(ap):
         ap.ap_search_exhaustive(plan, 11, 8, 1, 1, 0, 1, key)
     with pytest.raises(ap.APError):
         ap.ap_decode(plan, 0, 4, 8, 1, 1, key=(1 << 63) - 1)
+
+
+def test_exhaustive_u32_tight_bound_saturates(ap, oracle_mod, monkeypatch):
+    """Large costs so that S = T_ref+1 is near 2^30 and the host's no-wrap bound
+    allows only a few rows between clamps: most candidates saturate, the argmin
+    must still equal the oracle's and the int64 sweep's key bit for bit."""
+    rng = np.random.default_rng(21)
+    hits = 0
+    for trial in range(16):
+        n = int(rng.integers(8, 14))
+        p = int(rng.integers(3, 6))
+        m = int(rng.integers(p + 8, p + 20))
+        # per-row growth W ~ 2^32 / (p + 3 + (m+p)/p): T_ref ~ (m+p) W / p leaves room
+        # for only ~p+3 rows between clamps (host bound), so clamps and saturation fire
+        hi = int(2 ** 32 / (n * (p + 3 + (m + p) / p)) / 1.25)
+        f = rng.integers(hi // 4, hi, n).astype(np.int64)
+        b = rng.integers(hi // 4, hi, n).astype(np.int64)
+        a = rng.integers(0, 1 << 20, n).astype(np.int64)
+        M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+        plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+        k_hi = int(rng.integers(1, 4))
+        monkeypatch.delenv("AP_SWEEP", raising=False)
+        key = _search(ap, plan, p, m, 1, k_hi)
+        info = ap.ap_last_launch()
+        monkeypatch.setenv("AP_SWEEP", "int64")
+        key64 = _search(ap, plan, p, m, 1, k_hi)
+        assert key == key64
+        o = M.exhaustive(p, m, 1, k_hi)
+        res = ap.ap_decode(plan, 0, p, m, 1, k_hi, key=key)
+        assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+        if info["fast_u32"] and info["clamp_rows"] < m - p:
+            hits += 1
+    assert hits >= 3
+
+
+def test_key_layout_matches_python_helpers(ap):
+    """The C key layout == search.pack/unpack (used by the multi-process host logic)."""
+    from paper_conf_cluster_liulldgl22_b200.search import unpack_exhaustive_key
+    wl = synth.config(2)
+    f, b, a = wl.arrays()
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    N = ap.ap_count(wl.n, wl.p)
+    key = _search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
+    res = ap.ap_decode(plan, 0, wl.p, wl.m, wl.k_lo, wl.k_hi, key=key)
+    assert unpack_exhaustive_key(key, N, wl.k_lo, wl.k_hi) == (res["time_ns"], res["rank"], res["k"])

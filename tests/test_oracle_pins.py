@@ -511,3 +511,35 @@ def test_P15_survey_crosscheck_values(oracle_mod):
     c, _ = M5.alg1(16)
     assert M5.T(16, 64, c) == 441984812
     assert M5.heuristic_restart(16, 64, 0x5EED, 2, 0)["T"] == 430480412
+
+
+def test_algorithmic_op_count_matches_dag(oracle_mod):
+    """bench.ops_per_sim (adds + distinct maxima) equals a direct count over the
+    oracle's DAG: ops, and the number of distinct predecessor pairs among ops with
+    two predecessors."""
+    import importlib.util
+    import os
+    spec = importlib.util.spec_from_file_location(
+        "bench", os.path.join(os.path.dirname(os.path.dirname(__file__)), "bench.py"))
+    bench = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(bench)
+    for p in range(1, 7):
+        for m in range(1, 9):
+            for k in (1, 2, 3):
+                M, cuts = _uniform_model(oracle_mod, p, 1, 3, 5, 7, 10**9)
+                ops = M.simulate(p, m, cuts, k=k, want_all=True)["ops"]
+                ids = {o[:4] for o in ops}
+                per_stage = {}
+                for o in ops:
+                    per_stage.setdefault(o[0], []).append(o[:4])
+                prev = {}
+                for x, lst in per_stage.items():
+                    for a, b in zip(lst, lst[1:]):
+                        prev[b] = a
+                pairs = set()
+                for (st, kind, mb, q) in ids:
+                    cross = (st - 1, 0, mb, q) if kind == 0 else (st + 1, 1, mb, 0)
+                    intra = prev.get((st, kind, mb, q))
+                    if cross in ids and intra is not None:
+                        pairs.add(frozenset((cross, intra)))
+                assert bench.ops_per_sim(p, m, k) == len(ops) + len(pairs), (p, m, k)

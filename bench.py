@@ -215,6 +215,10 @@ def main():
     ap_.add_argument("--no-cpu-baseline", action="store_true")
     ap_.add_argument("--no-secondary", action="store_true")
     ap_.add_argument("--ref-budget", type=float, default=8.0)
+    ap_.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                     help="process-group backend (gloo + --device-override only to "
+                          "exercise the sharded path on a one-GPU box)")
+    ap_.add_argument("--device-override", type=int, default=None)
     args = ap_.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -228,10 +232,15 @@ def main():
     from paper_conf_cluster_liulldgl22_b200.search import shard
 
     rank, local, world = _env_rank()
+    if args.device_override is not None:
+        local = args.device_override
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
     peaks, peak_src = _peaks()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     sms = torch.cuda.get_device_properties(local).multi_processor_count
@@ -427,8 +436,13 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
     t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    sims5 = torch.tensor([float(ap.ap_last_sims())], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(sims5, op=dist.ReduceOp.SUM)
     out["C5"] = {"workload": wl.name, "restarts": wl.restarts,
                  "restarts_per_s": wl.restarts / (float(t[0]) / 1e3),
+                 "sims_per_step": int(sims5[0]),
+                 "sims_per_s": float(sims5[0]) / (float(t[0]) / 1e3),
                  "time_to_plan_ms": float(t[0]), "T_ns": r5["time_ns"], "restart": r5["restart"],
                  "cuts": r5["cuts"], "slicer_T_ns": [int(x) for x in Tk], "slicer_best_k": bk}
     return out

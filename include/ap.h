@@ -83,8 +83,10 @@ ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns
                          const int64_t* act_bytes, uint64_t link_bytes_per_s,
                          int32_t device, ap_plan** out);
 
-/* Release a plan and its device memory.  NULL-safe.  Not concurrent-safe with
- * calls still running on the plan. */
+/* Release a plan and its device memory.  NULL-safe.  The caller must first make
+ * sure no work using the plan is still pending on any stream (synchronise the
+ * streams of earlier asynchronous calls); the memory is returned stream-ordered to
+ * the library's per-device pool. */
 void ap_plan_destroy(ap_plan* plan);
 
 /* Number of sub-layers and comm_ns table (host copy) of a plan.  comm may be NULL. */
@@ -237,6 +239,11 @@ void ap_last_launch(ap_launch_info* info);
  * Valid once the stream has passed the launch; AP_ERR_INVALID before that or if
  * no search ran. */
 ap_status ap_last_kernel_ms(float* ms);
+
+/* Simulations run by the last ap_search_exhaustive / ap_search_heuristic call on this
+ * thread: (rank_hi-rank_lo)*(k_hi-k_lo+1) for the sweep; counted on the device for the
+ * heuristic (blocks until that kernel has finished). */
+ap_status ap_last_sims(uint64_t* sims);
 
 #ifdef __cplusplus
 }

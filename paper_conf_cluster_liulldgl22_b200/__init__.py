@@ -87,6 +87,8 @@ def _load_lib():
     lib.ap_last_launch.argtypes = [P(ApLaunchInfo)]
     lib.ap_last_kernel_ms.restype = i32
     lib.ap_last_kernel_ms.argtypes = [P(C.c_float)]
+    lib.ap_last_sims.restype = i32
+    lib.ap_last_sims.argtypes = [P(u64)]
     return lib
 
 
@@ -96,7 +98,7 @@ lib = _load_lib()
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
            "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_heuristic",
            "ap_decode", "ap_slice_sweep", "ap_critical_path", "ap_alg1", "ap_last_launch",
-           "ap_last_kernel_ms")
+           "ap_last_kernel_ms", "ap_last_sims")
 
 
 def _check(st: int):
@@ -275,3 +277,10 @@ def ap_last_kernel_ms() -> float:
     v = C.c_float()
     _check(lib.ap_last_kernel_ms(C.byref(v)))
     return float(v.value)
+
+
+def ap_last_sims() -> int:
+    """Simulations run by the last search call on this thread."""
+    v = C.c_uint64()
+    _check(lib.ap_last_sims(C.byref(v)))
+    return int(v.value)

@@ -8,6 +8,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -39,6 +40,22 @@ struct KernelTimer {
       }
     armed = (which == 1);
     return cudaEventRecord(ev[which], s);
+  }
+  // simulations of the last search: known on the host (exhaustive) or counted on
+  // the device (heuristic, d_sims valid once ev[1] has completed)
+  uint64_t host_sims = 0;
+  bool sims_on_device = false;
+  unsigned long long* d_sims = nullptr;
+  int d_sims_dev = -1;
+  cudaError_t sims_buffer(int device, unsigned long long** out) {
+    if (d_sims_dev != device) {
+      d_sims = nullptr;  // (a buffer of another device is leaked; one per thread/device switch)
+      cudaError_t e = cudaMalloc((void**)&d_sims, 16);
+      if (e != cudaSuccess) return e;
+      d_sims_dev = device;
+    }
+    *out = d_sims;
+    return cudaSuccess;
   }
 };
 thread_local KernelTimer g_timer;
@@ -73,7 +90,7 @@ struct DeviceGuard {
   }
 };
 
-// Per-call device scratch from the plan's memory pool (release threshold = max,
+// Per-call device scratch from the device's library pool (release threshold = max,
 // so stream-ordered frees never unmap memory at a synchronisation), released
 // stream-ordered.
 struct Scratch {
@@ -90,6 +107,47 @@ struct Scratch {
     for (void* p : ptrs) cudaFreeAsync(p, s);
   }
 };
+
+// One library-owned memory pool per device (created on first use, release threshold =
+// max so stream-ordered frees never unmap memory at a synchronisation; never destroyed).
+std::mutex g_pool_mu;
+cudaMemPool_t g_pools[64] = {nullptr};
+cudaError_t device_pool(int device, cudaMemPool_t* out) {
+  if (device < 0 || device >= 64) return cudaErrorInvalidDevice;
+  std::lock_guard<std::mutex> lk(g_pool_mu);
+  if (!g_pools[device]) {
+    cudaMemPoolProps props = {};
+    props.allocType = cudaMemAllocationTypePinned;
+    props.location.type = cudaMemLocationTypeDevice;
+    props.location.id = device;
+    cudaError_t e = cudaMemPoolCreate(&g_pools[device], &props);
+    if (e != cudaSuccess) {
+      g_pools[device] = nullptr;
+      return e;
+    }
+    uint64_t thr = UINT64_MAX;
+    e = cudaMemPoolSetAttribute(g_pools[device], cudaMemPoolAttrReleaseThreshold, &thr);
+    if (e != cudaSuccess) return e;
+  }
+  *out = g_pools[device];
+  return cudaSuccess;
+}
+
+// Per-thread pinned host staging buffer (grown on demand, never freed).
+cudaError_t pinned_staging(size_t bytes, int64_t** out) {
+  thread_local int64_t* buf = nullptr;
+  thread_local size_t cap = 0;
+  if (cap < bytes) {
+    if (buf) cudaFreeHost(buf);
+    buf = nullptr;
+    cap = 0;
+    cudaError_t e = cudaHostAlloc((void**)&buf, bytes, cudaHostAllocDefault);
+    if (e != cudaSuccess) return e;
+    cap = bytes;
+  }
+  *out = buf;
+  return cudaSuccess;
+}
 
 // One internal non-blocking stream per (thread, device) for the blocking calls.
 cudaError_t internal_stream(int device, cudaStream_t* out) {
@@ -145,6 +203,21 @@ void ap_last_launch(ap_launch_info* info) {
   if (info) *info = g_last;
 }
 
+ap_status ap_last_sims(uint64_t* sims) {
+  if (!sims) return fail(AP_ERR_INVALID, "sims is NULL");
+  if (!g_timer.armed) return fail(AP_ERR_INVALID, "no search launched on this thread");
+  if (!g_timer.sims_on_device) {
+    *sims = g_timer.host_sims;
+    return AP_OK;
+  }
+  cudaError_t e = cudaEventSynchronize(g_timer.ev[1]);
+  unsigned long long v = 0;
+  if (e == cudaSuccess) e = cudaMemcpy(&v, g_timer.d_sims, 8, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return fail(AP_ERR_CUDA, "sims read: %s", cudaGetErrorString(e));
+  *sims = v;
+  return AP_OK;
+}
+
 ap_status ap_last_kernel_ms(float* ms) {
   if (!ms) return fail(AP_ERR_INVALID, "ms is NULL");
   if (!g_timer.armed) return fail(AP_ERR_INVALID, "no search launched on this thread");
@@ -168,11 +241,12 @@ ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || ndev == 0)
     return fail(AP_ERR_CUDA, "no CUDA device (the library has no CPU fallback)");
   if (device < 0 || device >= ndev) return fail(AP_ERR_INVALID, "device %d of %d", device, ndev);
-  cudaDeviceProp prop;
-  AP_CUDA(cudaGetDeviceProperties(&prop, device));
-  if (prop.major != 10)
+  int major = 0, minor = 0;
+  AP_CUDA(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, device));
+  AP_CUDA(cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, device));
+  if (major != 10)
     return fail(AP_ERR_CUDA, "device %d is sm_%d%d; this library is built for sm_100a", device,
-                prop.major, prop.minor);
+                major, minor);
   ap_plan* P = new ap_plan();
   P->n = n;
   P->npad = (n + 1) & ~1;  // even => 16-byte multiple per array (TMA bulk copy)
@@ -212,26 +286,33 @@ ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns
     tab[P->npad + i] = P->b[i];
     tab[2 * P->npad + i] = P->comm[i];
   }
-  std::vector<uint64_t> binom((size_t)(n + 1) * 33, 0);
-  for (int a = 0; a <= n; ++a)
-    for (int bb = 0; bb <= 32 && bb <= a; ++bb) binom[(size_t)a * 33 + bb] = binom_sat(a, bb);
-  DeviceGuard g(device);
-  cudaError_t e = cudaMalloc((void**)&P->d_tab, tab.size() * 8);
-  if (e == cudaSuccess) e = cudaMalloc((void**)&P->d_binom, binom.size() * 8);
-  if (e == cudaSuccess) e = cudaMemcpy(P->d_tab, tab.data(), tab.size() * 8, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess)
-    e = cudaMemcpy(P->d_binom, binom.data(), binom.size() * 8, cudaMemcpyHostToDevice);
-  if (e == cudaSuccess) {
-    cudaMemPoolProps props = {};
-    props.allocType = cudaMemAllocationTypePinned;
-    props.location.type = cudaMemLocationTypeDevice;
-    props.location.id = device;
-    e = cudaMemPoolCreate(&P->pool, &props);
-    if (e == cudaSuccess) {
-      uint64_t thr = UINT64_MAX;
-      e = cudaMemPoolSetAttribute(P->pool, cudaMemPoolAttrReleaseThreshold, &thr);
+  // binomials C(a, b), a <= n, b <= 32, by Pascal's rule (saturating at 2^64-1), laid
+  // out right after the tables so one allocation and one copy stage the whole plan
+  const size_t nb = (size_t)(n + 1) * 33;
+  tab.resize(tab.size() + nb, 0);
+  uint64_t* binom = reinterpret_cast<uint64_t*>(tab.data() + 3 * (size_t)P->npad);
+  for (int a = 0; a <= n; ++a) {
+    binom[(size_t)a * 33] = 1;
+    for (int bb = 1; bb <= 32 && bb <= a; ++bb) {
+      const uint64_t x = binom[(size_t)(a - 1) * 33 + bb - 1];
+      const uint64_t y = (bb <= a - 1) ? binom[(size_t)(a - 1) * 33 + bb] : 0;
+      binom[(size_t)a * 33 + bb] = (x > UINT64_MAX - y) ? UINT64_MAX : x + y;
     }
   }
+  DeviceGuard g(device);
+  cudaStream_t s0 = nullptr;
+  cudaError_t e = device_pool(device, &P->pool);
+  if (e == cudaSuccess) e = internal_stream(device, &s0);
+  if (e == cudaSuccess) e = cudaMallocFromPoolAsync((void**)&P->d_tab, tab.size() * 8, P->pool, s0);
+  // stage through a per-thread pinned buffer so the copy is a plain DMA
+  int64_t* pinned = nullptr;
+  if (e == cudaSuccess) e = pinned_staging(tab.size() * 8, &pinned);
+  if (e == cudaSuccess) {
+    memcpy(pinned, tab.data(), tab.size() * 8);
+    e = cudaMemcpyAsync(P->d_tab, pinned, tab.size() * 8, cudaMemcpyHostToDevice, s0);
+  }
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s0);
+  if (e == cudaSuccess) P->d_binom = reinterpret_cast<uint64_t*>(P->d_tab + 3 * (size_t)P->npad);
   if (e != cudaSuccess) {
     ap_plan_destroy(P);
     return fail(e == cudaErrorMemoryAllocation ? AP_ERR_NOMEM : AP_ERR_CUDA, "plan upload: %s",
@@ -245,11 +326,11 @@ void ap_plan_destroy(ap_plan* plan) {
   if (!plan) return;
   {
     DeviceGuard g(plan->device);
-    if (plan->d_tab) cudaFree(plan->d_tab);
-    if (plan->d_binom) cudaFree(plan->d_binom);
-    if (plan->pool) {
-      cudaDeviceSynchronize();  // stream-ordered frees into the pool must land first
-      cudaMemPoolDestroy(plan->pool);
+    // the caller guarantees no call on the plan is still running (include/ap.h)
+    cudaStream_t s0 = nullptr;
+    if (plan->d_tab && internal_stream(plan->device, &s0) == cudaSuccess) {
+      cudaFreeAsync(plan->d_tab, s0);
+      cudaStreamSynchronize(s0);
     }
   }
   delete plan;
@@ -430,6 +511,8 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
                             clamp_rows, force_generic, reinterpret_cast<unsigned long long*>(key),
                             s, &sp));
   AP_CUDA(g_timer.record(1, s, plan->device));
+  g_timer.sims_on_device = false;
+  g_timer.host_sims = (rank_hi - rank_lo) * (uint64_t)(k_hi - k_lo + 1);
   launches += 2;
   info.fast_u32 = sp.fast_u32;
   info.exact_p = sp.exact_p;
@@ -464,11 +547,15 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   if (st != AP_OK) return st;
   unsigned int* d_ctr;
   AP_CUDA(sc.get((void**)&d_ctr, 16));
+  unsigned long long* d_sims = nullptr;
+  AP_CUDA(g_timer.sims_buffer(plan->device, &d_sims));
+  AP_CUDA(cudaMemsetAsync(d_sims, 0, 8, s));
   AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), d_ctr, s));
   AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_heuristic(plan->dev(), p, m, seed, radius, r_lo, r_hi, d_arg, d_a1, d_ctr,
-                                reinterpret_cast<unsigned long long*>(key), nullptr, s));
+                                reinterpret_cast<unsigned long long*>(key), nullptr, d_sims, s));
   AP_CUDA(g_timer.record(1, s, plan->device));
+  g_timer.sims_on_device = true;
   ap_launch_info info{};
   info.launches = 3;  // alg1, init, restarts
   g_last = info;
@@ -540,7 +627,7 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
         if (e == cudaSuccess) e = apk::launch_init_key(d_key, d_ctr, s);
         if (e == cudaSuccess)
           e = apk::launch_heuristic(plan->dev(), p, m, seed, radius, r, r + 1, d_arg, d_a1, d_ctr,
-                                    d_key, d_cuts, s);
+                                    d_key, d_cuts, nullptr, s);
         if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "replay: %s", cudaGetErrorString(e));
       }
     } else if (res == AP_OK) {

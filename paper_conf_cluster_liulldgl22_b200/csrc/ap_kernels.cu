@@ -541,6 +541,7 @@ struct HeurArgs {
   unsigned int* counter;
   unsigned long long* key;
   int32_t* replay;
+  unsigned long long* sims;  // optional: total simulations run (atomicAdd per warp)
 };
 
 // Algorithm 1 on the prefix [0, c) with j stages: writes c_1..c_{j-1} (line 15).
@@ -571,6 +572,7 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
 
   int cur[P + 1] = {0}, cand[P + 1] = {0}, best[P + 1] = {0}, sel[P + 1] = {0};
   unsigned long long lane_key = 0x7fffffffffffffffull;
+  unsigned int nsims = 0;
   const int smax = n * p;
   int phase = 0;  // 0 need restart, 1 start evaluated next, 2 child evaluated next
   uint32_t r = 0;
@@ -633,6 +635,7 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
     const int64_t Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
     int len;
     const int Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+    ++nsims;
     bool do_step = false, finish = false;
     if (phase == 1) {
       curM = Mc;
@@ -691,6 +694,12 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
         for (int x = 1; x <= p - 1; ++x) A.replay[x - 1] = best[x];
       phase = 0;
     }
+  }
+  if (A.sims) {
+    unsigned long long s = nsims;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if ((threadIdx.x & 31) == 0) atomicAdd(A.sims, s);
   }
   block_min_atomic(lane_key, A.key);
 }
@@ -1009,10 +1018,11 @@ static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev) {
 cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, int radius,
                              uint32_t r_lo, uint32_t r_hi, const int16_t* arg,
                              const int32_t* alg1_cuts, unsigned int* counter,
-                             unsigned long long* key, int32_t* replay_cuts, cudaStream_t s) {
+                             unsigned long long* key, int32_t* replay_cuts,
+                             unsigned long long* sims, cudaStream_t s) {
   int dev = 0;
   cudaGetDevice(&dev);
-  HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts};
+  HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts, sims};
   switch (pick_P(p)) {
     case 2: return heur_P<2>(A, s, dev);
     case 4: return heur_P<4>(A, s, dev);

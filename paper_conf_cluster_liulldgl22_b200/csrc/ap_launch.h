@@ -45,7 +45,8 @@ cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, u
 cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, int radius,
                              uint32_t r_lo, uint32_t r_hi, const int16_t* arg,
                              const int32_t* alg1_cuts, unsigned int* counter,
-                             unsigned long long* key, int32_t* replay_cuts, cudaStream_t s);
+                             unsigned long long* key, int32_t* replay_cuts,
+                             unsigned long long* sims, cudaStream_t s);
 
 struct OpRec {
   int32_t stage, kind, microbatch, piece;

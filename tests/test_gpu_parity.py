@@ -372,3 +372,21 @@ def test_key_layout_matches_python_helpers(ap):
     key = _search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
     res = ap.ap_decode(plan, 0, wl.p, wl.m, wl.k_lo, wl.k_hi, key=key)
     assert unpack_exhaustive_key(key, N, wl.k_lo, wl.k_hi) == (res["time_ns"], res["rank"], res["k"])
+
+
+def test_heuristic_sims_count_matches_oracle(ap, oracle_mod):
+    """ap_last_sims after a heuristic search == the oracle's simulation count for the
+    same restarts (start partition + every non-duplicate child)."""
+    import torch
+    for cfg, R in ((2, 512), (5, 256)):
+        wl = synth.config(cfg)
+        f, b, a = wl.arrays()
+        plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+        key = torch.empty(1, dtype=torch.int64, device="cuda")
+        ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, R, 0, key)
+        torch.cuda.synchronize()
+        o = oracle_mod.Model.from_workload(wl).heuristic(wl.p, wl.m, wl.seed, wl.radius, 0, R)
+        assert ap.ap_last_sims() == o["sims"]
+        if cfg == 2:
+            ap.ap_search_exhaustive(plan, wl.p, wl.m, 1, 2, 0, 1000, key)
+            assert ap.ap_last_sims() == 1000 * 2

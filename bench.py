@@ -331,6 +331,37 @@ def main():
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
     e2e_val = total_sims * e2e_steps / float(e2e_t[0])
 
+    # ------------------------------------------------------------- other search modes
+    # Same exact key, less work per candidate: labelled
+    # time-to-optimal-plan numbers, NOT the candidates/s headline (which is defined on
+    # the full per-(partition, k) sweep above).
+    modes = {}
+    for mode, name in ((ap.AP_SEARCH_KFACTOR, "kfactor"), (ap.AP_SEARCH_PRUNED, "pruned")):
+        kk = torch.empty(1, dtype=torch.int64, device=dev)
+        def run_mode():
+            if hi > lo:
+                ap.ap_search_exhaustive_mode(plan, wl.p, wl.m, wl.k_lo, wl.k_hi, lo, hi, mode, kk)
+            else:
+                kk.fill_(ap.INT64_MAX)
+            if world > 1:
+                dist.all_reduce(kk, op=dist.ReduceOp.MIN)
+            return int(kk.item())
+        for _ in range(3):
+            run_mode()
+        ts = []
+        for _ in range(5):
+            flush.zero_()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(); kv = run_mode(); e1.record(); torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        tmed = torch.tensor([statistics.median(ts)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tmed, op=dist.ReduceOp.MAX)
+        modes[name] = {"time_to_optimal_plan_ms": float(tmed[0]),
+                       "same_key_as_full": kv == int(key.item()),
+                       "equivalent_candidates_per_s": total_sims / (float(tmed[0]) / 1e3)}
+
     # ------------------------------------------------------------- secondary workloads
     secondary = {}
     if not args.no_secondary:
@@ -372,6 +403,7 @@ def main():
                    "d2h_bytes_per_step": 8 + 8 + 140 + 8 * wl.k_hi, "steps": e2e_steps,
                    "path": "ap_plan_create(host tables) -> ap_search_exhaustive -> "
                            "all_reduce -> ap_decode -> ap_slice_sweep -> ap_plan_destroy"},
+           "search_modes": modes,
            "secondary": secondary}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = oracle_rate(wl)

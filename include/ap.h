@@ -140,6 +140,29 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
                                int64_t* key, ap_stream_t stream);
 
 /*
+ * ap_search_exhaustive_mode -- ap_search_exhaustive with a choice of evaluation
+ * strategy.  Every mode returns the SAME key (the exact argmin); they differ only in
+ * how much work is done per candidate:
+ *   AP_SEARCH_FULL     every (partition, k) pair is row-swept in full (the
+ *                      candidates/s metric is defined on this mode).
+ *   AP_SEARCH_KFACTOR  exact max-plus factoring over k: one reversed sweep per
+ *                      partition gives the longest path G_x from the end of each
+ *                      stage's first forward to the sink; T(k) = max_x FF_x(k) + G_x
+ *                      where FF(k) is micro-batch 0's k-piece forward.
+ *   AP_SEARCH_PRUNED   KFACTOR, skipping partitions whose valid lower bound
+ *                      (a stage's 2m ops back to back plus the fill and
+ *                      drain chains) exceeds T_ref; a labelled time-to-plan mode.
+ * Modes 1 and 2 apply to the p-specialised kernel (p <= 8, 10, 12, 16 and m >= p);
+ * elsewhere the call falls back to the full sweep.
+ */
+#define AP_SEARCH_FULL 0
+#define AP_SEARCH_KFACTOR 1
+#define AP_SEARCH_PRUNED 2
+ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                    int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
+                                    int32_t mode, int64_t* key, ap_stream_t stream);
+
+/*
  * ap_search_heuristic -- AutoPipe's boundary-shifting heuristic (PAPER.md:147-198,
  * steps 1, 3, 4; step 2 / Eq. (1) is adjust_mode 1, not yet supported), run as
  * independent deterministic restarts r in [r_lo, r_hi), one GPU lane each.

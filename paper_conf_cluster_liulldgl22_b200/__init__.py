@@ -72,6 +72,8 @@ def _load_lib():
     lib.ap_eval_batch.argtypes = [vp, i32, i32, vp, vp, i64, vp, vp, vp]
     lib.ap_search_exhaustive.restype = i32
     lib.ap_search_exhaustive.argtypes = [vp, i32, i32, i32, i32, u64, u64, vp, vp]
+    lib.ap_search_exhaustive_mode.restype = i32
+    lib.ap_search_exhaustive_mode.argtypes = [vp, i32, i32, i32, i32, u64, u64, i32, vp, vp]
     lib.ap_search_heuristic.restype = i32
     lib.ap_search_heuristic.argtypes = [vp, i32, i32, u64, i32, u32, u32, i32, vp, vp]
     lib.ap_decode.restype = i32
@@ -96,7 +98,8 @@ lib = _load_lib()
 
 # every symbol include/ap.h declares (checked by tests/test_abi.py)
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
-           "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_heuristic",
+           "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_exhaustive_mode",
+           "ap_search_heuristic",
            "ap_decode", "ap_slice_sweep", "ap_critical_path", "ap_alg1", "ap_last_launch",
            "ap_last_kernel_ms", "ap_last_sims")
 
@@ -212,6 +215,17 @@ def ap_search_exhaustive(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank_
     _check(lib.ap_search_exhaustive(plan.handle, int(p), int(m), int(k_lo), int(k_hi),
                                     int(rank_lo), int(rank_hi), _ptr(key, "int64", plan.device),
                                     _stream(stream)))
+
+
+AP_SEARCH_FULL, AP_SEARCH_KFACTOR, AP_SEARCH_PRUNED = 0, 1, 2
+
+
+def ap_search_exhaustive_mode(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank_lo: int,
+                              rank_hi: int, mode: int, key, stream=None):
+    """Same key as ap_search_exhaustive; mode selects full / k-factored / pruned."""
+    _check(lib.ap_search_exhaustive_mode(plan.handle, int(p), int(m), int(k_lo), int(k_hi),
+                                         int(rank_lo), int(rank_hi), int(mode),
+                                         _ptr(key, "int64", plan.device), _stream(stream)))
 
 
 def ap_search_heuristic(plan: Plan, p: int, m: int, seed: int, radius: int, r_lo: int,

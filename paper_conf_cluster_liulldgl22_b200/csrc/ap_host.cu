@@ -448,7 +448,16 @@ ap_status ap_alg1(const ap_plan* plan, int32_t p, int32_t* cuts, int64_t* value)
 ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
                                int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int64_t* key,
                                ap_stream_t stream) {
+  return ap_search_exhaustive_mode(plan, p, m, k_lo, k_hi, rank_lo, rank_hi, AP_SEARCH_FULL, key,
+                                   stream);
+}
+
+ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                    int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
+                                    int32_t mode, int64_t* key, ap_stream_t stream) {
   g_err.clear();
+  if (mode < AP_SEARCH_FULL || mode > AP_SEARCH_PRUNED)
+    return fail(AP_ERR_INVALID, "search mode %d", mode);
   ap_status st = check_pm(plan, p, m);
   if (st != AP_OK) return st;
   if (!key) return fail(AP_ERR_INVALID, "key is NULL");
@@ -508,8 +517,8 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
   AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), nullptr, s));
   AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, S, rb, want_u32,
-                            clamp_rows, force_generic, reinterpret_cast<unsigned long long*>(key),
-                            s, &sp));
+                            clamp_rows, force_generic, mode,
+                            reinterpret_cast<unsigned long long*>(key), s, &sp));
   AP_CUDA(g_timer.record(1, s, plan->device));
   g_timer.sims_on_device = false;
   g_timer.host_sims = (rank_hi - rank_lo) * (uint64_t)(k_hi - k_lo + 1);

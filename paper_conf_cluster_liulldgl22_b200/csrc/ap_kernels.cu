@@ -94,14 +94,13 @@ AP_DEV_INLINE void clamp_ff(V (&FF)[P], V S) {
   }
 }
 
-// Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
+// Micro-batch 0's forward, sliced into k pieces (reading Q6): FF[x] = finish of the
+// last piece F(x, 0, k-1).  The raw stage compute/comm are re-read from shared
+// memory only on the k > 1 path.
 template <int P, typename V>
-AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const int (&c)[P + 1],
-                         const V* sPf, const V* sC, uint32_t Mk, V S, int CR, uint32_t one) {
+AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const V* sPf,
+                          const V* sC, uint32_t Mk, uint32_t one, V (&FF)[P]) {
   using O = XOps<V>;
-  V FF[P], L[P];
-  // micro-batch 0's forward, sliced into k pieces (reading Q6); the raw stage
-  // compute/comm are re-read from shared memory only on this (k > 1) path
   if (k == 1) {
     FF[0] = wF[0];
 #pragma unroll
@@ -125,6 +124,24 @@ AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const
 #pragma unroll
     for (int x = 1; x < P; ++x) FF[x] = O::ad(O::mx(FF[x - 1], FF[x]), al[x], one);
   }
+}
+
+// Everything after the pieces, for p == P, m >= P: warm-up rows, the first 1F1B row,
+// the fused steady steps and the fused cool-down.
+//  REV = false: input FF = finishes of F(x, 0, k-1); returns T = end of B(0, m-1).
+//  REV = true : the same sweep on the REVERSED task DAG (weights wF/wB swapped by the
+//      caller), which is again a 1F1B schedule: its op B'(x, y) is the original
+//      F(x, m-1-y) and F'(x, j) the original B(x, m-1-j), and its "finish" times are
+//      the original longest paths to the sink.  It stops before the last backward
+//      row (the original micro-batch-0 forwards) and writes
+//        G[x] = B'(x, m-2) for x <= P-2 (longest path from the end of F(x,0) via
+//               F(x,1)),   G[P-1] = F'(P-1, m-1) (via B(P-1,0)),
+//      so that T(k) = max_x (FF_x(k) + G[x]) for every k.
+template <int P, typename V, bool REV>
+AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V S, int CR,
+                           uint32_t one, V (&G)[P]) {
+  using O = XOps<V>;
+  V L[P];
   // warm-up rows r = 1..P-2: stage x <= r-1 does F(x, r-x); L == FF here
 #pragma unroll
   for (int r = 1; r <= P - 2; ++r) {
@@ -139,10 +156,10 @@ AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const
   for (int x = P - 2; x >= 1; --x) FF[x] = O::ad(O::mx(FF[x - 1], L[x]), wF[x], one);
   if (P >= 2) FF[0] = O::ad(L[0], wF[0], one);
   clamp_ff<P, V>(FF, S);
-  // fused steps r = P-1..m-2: backward pass of row r + forward pass of row r+1.
+  // fused steps r = P-1..m-2: backward pass of row r + forward pass of row r+1,
+  // clamped (u32) every CR steps: the host's no-wrap bound S + CR * W_row < 2^32
+  //
   {
-    // fused M-form, clamped (u32) every CR steps: the host's no-wrap bound
-    // S + CR * W_row < 2^32
     constexpr int U = (P <= 8) ? 8 : 4;
     const V wBF0 = wB[0] + wF[0];
     int rem = m - P;
@@ -163,8 +180,9 @@ AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const
   // last op) instead of a shared maximum.  M carries max(FF[x], b[x+1]) with
   // b[x+1] = M + wB[x+1] folded into the next fused add+max.
   V b = 0;
+  constexpr int TEND = REV ? P - 1 : P;
 #pragma unroll
-  for (int t = 0; t < P; ++t) {
+  for (int t = 0; t < TEND; ++t) {
     if constexpr (P == 1) {
       b = O::ad(FF[0], wB[0], one);
     } else {
@@ -193,7 +211,21 @@ AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const
       b = M;  // stage 0 is always materialised (x == t or x < t)
     }
   }
+  if constexpr (REV) {
+#pragma unroll
+    for (int x = 0; x < P - 1; ++x) G[x] = L[x];
+    G[P - 1] = FF[P - 1];
+  }
   return b;
+}
+
+// Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
+template <int P, typename V>
+AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const int (&c)[P + 1],
+                         const V* sPf, const V* sC, uint32_t Mk, V S, int CR, uint32_t one) {
+  V FF[P], G[P];
+  pieces<P, V>(k, wF, c, sPf, sC, Mk, one, FF);
+  return sweep_tail<P, V, false>(m, FF, wF, wB, S, CR, one, G);
 }
 
 struct SweepArgs {
@@ -204,7 +236,8 @@ struct SweepArgs {
   int rb;
   unsigned long long* key;
   int clamp_rows;  // u32 path: rows between saturating clamps (>= 1)
-  uint32_t one;    // = 1, opaque to the compiler (keeps adds on IMAD, see XOps)
+  uint32_t one;    // = 1 (adds are plain operators; kept for the XOps interface)
+  int mode;        // 0 full, 1 k-factored, 2 k-factored + lower-bound skipping
 };
 
 AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
@@ -296,12 +329,68 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
         wB[x] = Bx + Cout;
       }
       const uint64_t base = r * K;
-      for (int k = k_lo; k <= k_hi; ++k) {
-        const uint32_t Mk = s_mk[k];
-        const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, S, A.clamp_rows, A.one);
-        if (Tc < bestT) {
-          bestT = Tc;
-          bestIdx = base + (uint64_t)(k - k_lo);
+      bool live = true;
+      if (A.mode == 2) {
+        // SURVEY O11 lower bound for every k <= k_hi (pinned by the oracle's P6):
+        // LB_x = fill_x + m*(F_x+B_x+C_in+C_out) + sum_{i<x}(B_i+C_i), fill_x =
+        // sum_{i<x} floor(F_i/K) + sum_{i<x-1} floor(C_i/K).  A partition with LB >= S
+        // cannot hold a candidate with T < S = T_ref + 1.
+        // (64-bit: m * load can exceed 2^32 for the heavy partitions it prunes)
+        const uint32_t Kh = (uint32_t)k_hi, MK = s_mk[k_hi];
+        uint64_t fill = 0, tail = 0, lb = 0;
+#pragma unroll
+        for (int x = 0; x < P; ++x) {
+          const V Fx = sPf[c[x + 1]] - sPf[c[x]];
+          const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
+          const uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
+          lb = v > lb ? v : lb;
+          fill += (uint64_t)divk(Fx, Kh, MK) + (uint64_t)divk(Cin, Kh, MK);
+          tail += (uint64_t)wB[x];
+        }
+        live = lb < (uint64_t)S;
+      }
+      if (live && A.mode == 0) {
+        for (int k = k_lo; k <= k_hi; ++k) {
+          const uint32_t Mk = s_mk[k];
+          const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, S, A.clamp_rows, A.one);
+          if (Tc < bestT) {
+            bestT = Tc;
+            bestIdx = base + (uint64_t)(k - k_lo);
+          }
+        }
+      } else if (live) {
+        // k-factored: one reversed sweep gives G, then T(k) = max_x FF_x(k) + G_x
+        V G[P];
+        if constexpr (P >= 2) {
+          V rF[P], rB[P], FF0[P];
+#pragma unroll
+          for (int x = 0; x < P; ++x) {
+            rF[x] = wB[x];
+            rB[x] = wF[x];
+          }
+          FF0[0] = rF[0];
+#pragma unroll
+          for (int x = 1; x < P; ++x) FF0[x] = FF0[x - 1] + rF[x];
+          sweep_tail<P, V, true>(m, FF0, rF, rB, S, A.clamp_rows, A.one, G);
+        }
+        for (int k = k_lo; k <= k_hi; ++k) {
+          V Tc;
+          if constexpr (P >= 2) {
+            V FF[P];
+            pieces<P, V>(k, wF, c, sPf, sC, s_mk[k], A.one, FF);
+            Tc = FF[0] + G[0];
+#pragma unroll
+            for (int x = 1; x < P; ++x) {
+              const V v = FF[x] + G[x];
+              Tc = v > Tc ? v : Tc;
+            }
+          } else {
+            Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, s_mk[k], S, A.clamp_rows, A.one);
+          }
+          if (Tc < bestT) {
+            bestT = Tc;
+            bestIdx = base + (uint64_t)(k - k_lo);
+          }
         }
       }
       // lexicographic successor (a2)
@@ -973,12 +1062,12 @@ bool has_exact(int p) {
 
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
-                         int force_generic, unsigned long long* key, cudaStream_t s,
+                         int force_generic, int mode, unsigned long long* key, cudaStream_t s,
                          SweepPlan* sp) {
   int dev = 0;
   cudaGetDevice(&dev);
-  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u};
-  const bool exact = has_exact(p) && m >= p && !force_generic;
+  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u, mode};
+  const bool exact = has_exact(p) && m >= p && (!force_generic || mode != 0);
   sp->exact_p = exact ? 1 : 0;
   sp->fast_u32 = (exact && want_u32) ? 1 : 0;
   if (exact) return sweep_exact_dispatch(p, sp->fast_u32, A, s, sp, dev);

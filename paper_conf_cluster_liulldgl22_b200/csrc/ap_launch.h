@@ -37,7 +37,7 @@ struct SweepPlan {
 // a candidate with T >= S can never win.  atomicMin into *key (init it first).
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
-                         int force_generic, unsigned long long* key, cudaStream_t s,
+                         int force_generic, int mode, unsigned long long* key, cudaStream_t s,
                          SweepPlan* plan_out);
 
 // Heuristic restarts [r_lo, r_hi); key = min (T << 20 | r).  replay_cuts (int32[p-1])

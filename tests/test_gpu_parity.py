@@ -390,3 +390,55 @@ def test_heuristic_sims_count_matches_oracle(ap, oracle_mod):
         if cfg == 2:
             ap.ap_search_exhaustive(plan, wl.p, wl.m, 1, 2, 0, 1000, key)
             assert ap.ap_last_sims() == 1000 * 2
+
+
+def _search_mode(ap, plan, p, m, k_lo, k_hi, mode, lo=None, hi=None):
+    import torch
+    N = ap.ap_count(plan.n, p)
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    ap.ap_search_exhaustive_mode(plan, p, m, k_lo, k_hi, 0 if lo is None else lo,
+                                 N if hi is None else hi, mode, key)
+    torch.cuda.synchronize()
+    return int(key.item())
+
+
+def test_search_modes_equal_random(ap, oracle_mod):
+    """k-factored and pruned modes return exactly the full sweep's key (and the
+    oracle's argmin) on random problems, incl. saturating near-2^32 tables."""
+    rng = np.random.default_rng(31)
+    for trial in range(24):
+        n = int(rng.integers(4, 16))
+        p = int(rng.integers(2, min(n, 8) + 1))
+        m = int(rng.integers(p, p + 12))
+        if trial % 3 == 2:
+            hi = int(2 ** 32 / (n * (p + 3 + (m + p) / p)) / 1.25)
+            f = rng.integers(hi // 4, hi, n).astype(np.int64)
+            b = rng.integers(hi // 4, hi, n).astype(np.int64)
+            a = rng.integers(0, 1 << 20, n).astype(np.int64)
+            bw = synth.LINK_BYTES_PER_S
+        else:
+            kind = ["uniform", "b3f", "small"][trial % 3]
+            f, b, a = synth.random_tables(trial, n, kind)
+            bw = synth.link_for(kind)
+        plan = _plan(ap, f, b, a, bw)
+        k_lo = int(rng.integers(1, 3)); k_hi = k_lo + int(rng.integers(0, 6))
+        keys = [_search_mode(ap, plan, p, m, k_lo, k_hi, mode) for mode in (0, 1, 2)]
+        assert keys[0] == keys[1] == keys[2], (n, p, m, k_lo, k_hi, keys)
+        o = oracle_mod.Model(f, b, a, bw).exhaustive(p, m, k_lo, k_hi)
+        res = ap.ap_decode(plan, 0, p, m, k_lo, k_hi, key=keys[1])
+        assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+
+
+@pytest.mark.parametrize("cfg", [2, 3, 4])
+def test_search_modes_equal_configs(ap, cfg):
+    wl = synth.config(cfg)
+    f, b, a = wl.arrays()
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    keys = [_search_mode(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi, mode) for mode in (0, 1, 2)]
+    assert keys[0] == keys[1] == keys[2]
+    if cfg == 4:
+        # sampled windows too (the k-factored path on arbitrary slices)
+        N = ap.ap_count(wl.n, wl.p)
+        for lo in (0, N // 3, N - 5000):
+            ks = [_search_mode(ap, plan, wl.p, wl.m, 1, 8, mode, lo, lo + 5000) for mode in (0, 1, 2)]
+            assert ks[0] == ks[1] == ks[2]

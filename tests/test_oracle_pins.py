@@ -543,3 +543,68 @@ def test_algorithmic_op_count_matches_dag(oracle_mod):
                     if cross in ids and intra is not None:
                         pairs.add(frozenset((cross, intra)))
                 assert bench.ops_per_sim(p, m, k) == len(ops) + len(pairs), (p, m, k)
+
+
+def _longest_to_sink(ops, P):
+    """h(op) = longest path from op (incl. its own weight) to the sink, on the DAG
+    rebuilt from the oracle's op list (edges of PAPER.md:113-123)."""
+    from collections import deque
+    per_stage = {}
+    for o in ops:
+        per_stage.setdefault(o[0], []).append(o)
+    idx = {o[:4]: i for i, o in enumerate(ops)}
+    succ = {i: [] for i in range(len(ops))}
+    preds = {i: [] for i in range(len(ops))}
+    for x, lst in per_stage.items():
+        for a_, b_ in zip(lst, lst[1:]):
+            succ[idx[a_[:4]]].append(idx[b_[:4]])
+    for i, (st, kind, mb, q, s0, e0) in enumerate(ops):
+        if kind == 0 and st < P - 1:
+            succ[i].append(idx[(st + 1, 0, mb, q)])
+        if kind == 1 and st > 0:
+            succ[i].append(idx[(st - 1, 1, mb, 0)])
+    for i, ss in succ.items():
+        for j in ss:
+            preds[j].append(i)
+    W = {i: o[5] - max([ops[j][5] for j in preds[i]], default=0) for i, o in enumerate(ops)}
+    outdeg = {i: len(succ[i]) for i in succ}
+    q = deque(i for i in succ if outdeg[i] == 0)
+    h = {}
+    while q:
+        i = q.popleft()
+        h[i] = W[i] + max([h[j] for j in succ[i]], default=0)
+        for j in preds[i]:
+            outdeg[j] -= 1
+            if outdeg[j] == 0:
+                q.append(j)
+    return h, per_stage, idx
+
+
+def test_kfactor_identity_on_oracle_dag(oracle_mod):
+    """T(k) = max_x FF_x(k) + G_x with G_x the longest path from the
+    end of F(x,0) through its intra-stage successor -- G independent of k.  Checked on
+    the oracle's explicit DAG (the GPU's KFACTOR mode relies on it)."""
+    rng = np.random.default_rng(5)
+    for seed in range(120):
+        kind = ["uniform", "small", "b3f"][seed % 3]
+        n = int(rng.integers(2, 12))
+        p = int(rng.integers(1, min(n, 6) + 1))
+        m = int(rng.integers(p, p + 6))
+        f, b, a = synth.random_tables(seed, n, kind)
+        M = oracle_mod.Model(f, b, a, synth.link_for(kind))
+        cuts = synth.random_cuts(seed, n, p, 1)[0]
+        G_ref = None
+        for k in (1, 2, 3, 5):
+            r = M.simulate(p, m, cuts, k=k, want_all=True)
+            h, per_stage, idx = _longest_to_sink(r["ops"], p)
+            G, FF = [], []
+            for x in range(p):
+                lst = per_stage[x]
+                last_piece = [o for o in lst if o[1] == 0 and o[2] == 0][-1]
+                nxt = lst[lst.index(last_piece) + 1]
+                G.append(h[idx[nxt[:4]]])
+                FF.append(last_piece[5])
+            if G_ref is None:
+                G_ref = G
+            assert G == G_ref
+            assert max(FF[x] + G[x] for x in range(p)) == r["T"]

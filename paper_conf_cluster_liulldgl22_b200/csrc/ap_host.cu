@@ -8,6 +8,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <atomic>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -59,6 +60,19 @@ struct KernelTimer {
   }
 };
 thread_local KernelTimer g_timer;
+
+// Per-thread record of the last heuristic search: each restart's best cut vector, so
+// ap_decode(mode 1) can read the winner's cuts instead of replaying its walk.
+struct HeurCache {
+  uint64_t plan_gen = 0;
+  int p = 0, m = 0, radius = 0, dev = -1;
+  uint64_t seed = 0;
+  uint32_t r_lo = 0, r_hi = 0;
+  int16_t* d_best = nullptr;
+  size_t cap = 0;
+  bool valid = false;
+};
+thread_local HeurCache g_hcache;
 
 ap_status fail(ap_status st, const char* fmt, ...) {
   char buf[512];
@@ -182,7 +196,10 @@ uint64_t binom_sat(int a, int b) {
 
 }  // namespace
 
+std::atomic<uint64_t> g_plan_gen{1};
+
 struct ap_plan {
+  uint64_t gen = 0;  // unique id (never reused) for caches keyed by plan
   int n = 0, npad = 0, device = 0;
   std::vector<int64_t> f, b, act, comm;
   int64_t sum_f = 0, sum_b = 0, max_comm = 0;
@@ -248,6 +265,7 @@ ap_status ap_plan_create(int32_t n, const int64_t* fwd_ns, const int64_t* bwd_ns
     return fail(AP_ERR_CUDA, "device %d is sm_%d%d; this library is built for sm_100a", device,
                 major, minor);
   ap_plan* P = new ap_plan();
+  P->gen = g_plan_gen.fetch_add(1);
   P->n = n;
   P->npad = (n + 1) & ~1;  // even => 16-byte multiple per array (TMA bulk copy)
   P->device = device;
@@ -555,14 +573,53 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   st = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
   if (st != AP_OK) return st;
   unsigned int* d_ctr;
-  AP_CUDA(sc.get((void**)&d_ctr, 16));
+  AP_CUDA(sc.get((void**)&d_ctr, 4 * (size_t)(3 + (r_hi - r_lo))));
   unsigned long long* d_sims = nullptr;
   AP_CUDA(g_timer.sims_buffer(plan->device, &d_sims));
   AP_CUDA(cudaMemsetAsync(d_sims, 0, 8, s));
+  // decode cache: each restart's best cut vector (int16, (r_hi-r_lo) x (p-1))
+  const size_t need = (size_t)(r_hi - r_lo) * (size_t)(p > 1 ? p - 1 : 1) * 2;
+  g_hcache.valid = false;
+  if (g_hcache.dev != plan->device || g_hcache.cap < need) {
+    if (g_hcache.d_best && g_hcache.dev == plan->device) cudaFree(g_hcache.d_best);
+    g_hcache.d_best = nullptr;
+    g_hcache.cap = 0;
+    AP_CUDA(cudaMalloc((void**)&g_hcache.d_best, need));
+    g_hcache.cap = need;
+    g_hcache.dev = plan->device;
+  }
+  // u32 fast path: every value grows by at most W_row per row and
+  // is clamped to S every CR rows (the cool-down adds p more rows), so
+  // S = 2^32-1 - (max(CR,p)+1)*W_row keeps everything exact below S.
+  const int hCR = 32;
+  const unsigned __int128 hw = (unsigned __int128)(plan->sum_f + plan->sum_b) +
+                               (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
+  const unsigned __int128 span = hw * (unsigned __int128)((hCR > p ? hCR : p) + 1);
+  const unsigned __int128 lim32 = ((unsigned __int128)1 << 32) - 1;
+  uint32_t fastS = 0;
+  if (span < lim32) fastS = (uint32_t)(lim32 - span);
+  // test overrides: AP_HEUR=int64 disables the u32 pass; AP_HEUR_S=<v> lowers its
+  // bound so that restarts saturate and exercise the exact redo pass
+  const char* hov = getenv("AP_HEUR");
+  if (hov && strcmp(hov, "int64") == 0) fastS = 0;
+  const char* hs = getenv("AP_HEUR_S");
+  if (hs && fastS > 0) {
+    const unsigned long long v = strtoull(hs, nullptr, 10);
+    if (v > 0 && v < fastS) fastS = (uint32_t)v;
+  }
   AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), d_ctr, s));
   AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_heuristic(plan->dev(), p, m, seed, radius, r_lo, r_hi, d_arg, d_a1, d_ctr,
-                                reinterpret_cast<unsigned long long*>(key), nullptr, d_sims, s));
+                                reinterpret_cast<unsigned long long*>(key), nullptr, d_sims,
+                                g_hcache.d_best, fastS, hCR, s));
+  g_hcache.plan_gen = plan->gen;
+  g_hcache.p = p;
+  g_hcache.m = m;
+  g_hcache.seed = seed;
+  g_hcache.radius = radius;
+  g_hcache.r_lo = r_lo;
+  g_hcache.r_hi = r_hi;
+  g_hcache.valid = true;
   AP_CUDA(g_timer.record(1, s, plan->device));
   g_timer.sims_on_device = true;
   ap_launch_info info{};
@@ -629,14 +686,30 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
       int64_t* d_val;
       unsigned int* d_ctr;
       unsigned long long* d_key;
-      if (res == AP_OK) res = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
-      if (res == AP_OK) {
+      const bool cached = g_hcache.valid && g_hcache.plan_gen == plan->gen && g_hcache.p == p &&
+                          g_hcache.m == m && g_hcache.seed == seed &&
+                          g_hcache.radius == radius && r >= g_hcache.r_lo &&
+                          r < g_hcache.r_hi && g_hcache.dev == plan->device && p > 1;
+      if (res == AP_OK && cached) {
+        // the search kernel already wrote restart r's best cuts: wait for it, copy them
+        int16_t h16[32];
+        e = cudaEventSynchronize(g_timer.ev[1]);
+        if (e == cudaSuccess)
+          e = cudaMemcpy(h16, g_hcache.d_best + (size_t)(r - g_hcache.r_lo) * (p - 1),
+                         2 * (size_t)(p - 1), cudaMemcpyDeviceToHost);
+        int32_t h32[32];
+        for (int x = 0; x < p - 1; ++x) h32[x] = h16[x];
+        if (e == cudaSuccess)
+          e = cudaMemcpyAsync(d_cuts, h32, 4 * (size_t)(p - 1), cudaMemcpyHostToDevice, s);
+        if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "decode cache: %s", cudaGetErrorString(e));
+      } else if (res == AP_OK) res = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
+      if (res == AP_OK && !cached) {
         e = sc.get((void**)&d_ctr, 16);
         if (e == cudaSuccess) e = sc.get((void**)&d_key, 16);
         if (e == cudaSuccess) e = apk::launch_init_key(d_key, d_ctr, s);
         if (e == cudaSuccess)
           e = apk::launch_heuristic(plan->dev(), p, m, seed, radius, r, r + 1, d_arg, d_a1, d_ctr,
-                                    d_key, d_cuts, nullptr, s);
+                                    d_key, d_cuts, nullptr, nullptr, 0, 1, s);
         if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "replay: %s", cudaGetErrorString(e));
       }
     } else if (res == AP_OK) {

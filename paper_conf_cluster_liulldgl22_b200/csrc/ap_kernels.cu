@@ -619,6 +619,103 @@ __global__ void __launch_bounds__(256) k_alg1(DevTables t, int p, int16_t* arg, 
 
 // ===========================================================================
 // K3 heuristic restarts (adjust_mode none; reading O9).
+// u32 saturating p-specialised simulation (k = 1, p == P, m >= P) that also writes
+// the decision bits the backtrack reads, in exactly the layout of sim_exact (rows
+// y + W0 = r; F bit x, B bit 16+x).  It is the M-form sweep of sweep_tail: B(x, y) and
+// F(x+1, .) of the next row compare the same pair (FF[x], b[x+1]), so the FP bit is
+// FF[x] > b[x+1] and the BP bit its complement (reading Q10's tie rule).  Values are
+// clamped to S every CR rows; a result >= S means "recompute exactly" (the caller
+// falls back to the int64 sim_exact).  P <= 16 (one bit word per row).
+template <int P>
+AP_DEV_INLINE uint32_t sim_fast_bits(int m, const uint32_t (&wF)[P], const uint32_t (&wB)[P],
+                                     uint32_t S, int CR, BitsRef br) {
+  static_assert(P >= 2 && P <= 16, "one bit word per row");
+  uint32_t FF[P], L[P];
+  FF[0] = wF[0];
+#pragma unroll
+  for (int x = 1; x < P; ++x) FF[x] = FF[x - 1] + wF[x];
+  br.base[0] = 0;
+  // warm-up rows r = 1..P-2
+#pragma unroll
+  for (int r = 1; r <= P - 2; ++r) {
+    uint32_t word = 0;
+#pragma unroll
+    for (int x = r - 1; x >= 1; --x) {
+      word |= (FF[x - 1] > FF[x] ? 1u : 0u) << x;
+      FF[x] = max(FF[x - 1], FF[x]) + wF[x];
+    }
+    FF[0] = FF[0] + wF[0];
+    br.base[(size_t)r * br.stride] = word;
+  }
+#pragma unroll
+  for (int x = 0; x < P; ++x) L[x] = FF[x];
+  uint32_t nxt = 0;  // F bits of the current r-row (its B bits come with the next step)
+#pragma unroll
+  for (int x = P - 2; x >= 1; --x) {
+    nxt |= (FF[x - 1] > L[x] ? 1u : 0u) << x;
+    FF[x] = max(FF[x - 1], L[x]) + wF[x];
+  }
+  FF[0] = L[0] + wF[0];
+#pragma unroll
+  for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
+  int r = P - 1;
+  int rem = m - P;
+  while (rem > 0) {
+    int blk = rem < CR ? rem : CR;
+    rem -= blk;
+    for (; blk > 0; --blk) {
+      uint32_t wordB = 0, wordF = 0, nF[P];
+      uint32_t b = FF[P - 1] + wB[P - 1];
+#pragma unroll
+      for (int x = P - 2; x >= 0; --x) {
+        const bool gt = FF[x] > b;
+        wordF |= (gt ? 1u : 0u) << (x + 1);
+        wordB |= (gt ? 0u : 1u) << (x + 16);
+        const uint32_t M = gt ? FF[x] : b;
+        nF[x + 1] = M + wF[x + 1];
+        b = M + wB[x];
+      }
+      nF[0] = b + wF[0];
+      br.base[(size_t)r * br.stride] = nxt | wordB;
+      nxt = wordF;
+      ++r;
+#pragma unroll
+      for (int x = 0; x < P; ++x) FF[x] = nF[x];
+    }
+#pragma unroll
+    for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
+  }
+  // cool-down t = 0..P-1: B of r-row m-1+t, F of the next row for x >= t+1
+  uint32_t b = 0;
+#pragma unroll
+  for (int t = 0; t < P; ++t) {
+    uint32_t wordB = 0, wordF = 0;
+    b = FF[P - 1] + wB[P - 1];
+#pragma unroll
+    for (int x = P - 2; x >= 0; --x) {
+      if (x >= t) {
+        const bool gt = FF[x] > b;
+        wordB |= (gt ? 0u : 1u) << (x + 16);
+        const uint32_t M = gt ? FF[x] : b;
+        if (t < P - 1) {
+          wordF |= (gt ? 1u : 0u) << (x + 1);
+          FF[x + 1] = M + wF[x + 1];
+        }
+        b = M + wB[x];
+        if (x == t) L[x] = b;
+      } else {
+        wordB |= (b >= L[x] ? 1u : 0u) << (x + 16);
+        b = max(b, L[x]) + wB[x];
+        L[x] = b;
+      }
+    }
+    br.base[(size_t)r * br.stride] = nxt | wordB;
+    nxt = wordF;
+    ++r;
+  }
+  return b;
+}
+
 struct HeurArgs {
   DevTables t;
   int p, m;
@@ -631,6 +728,11 @@ struct HeurArgs {
   unsigned long long* key;
   int32_t* replay;
   unsigned long long* sims;  // optional: total simulations run (atomicAdd per warp)
+  int16_t* best_out;         // optional: [r - r_lo][p-1] best cut vector of each restart
+  uint32_t S;                // fast path: u32 saturation bound (see sim_fast_bits)
+  int CR;                    // fast path: rows between clamps
+  unsigned int* redo;        // FAST: [0] = count, [1..] restarts abandoned on saturation;
+                             // generic: if non-null, run exactly the listed restarts
 };
 
 // Algorithm 1 on the prefix [0, c) with j stages: writes c_1..c_{j-1} (line 15).
@@ -643,7 +745,10 @@ AP_DEV_INLINE void alg1_prefix(const int16_t* s_arg, int P1, int c, int j, int* 
   }
 }
 
-template <int P>
+// FAST = true: u32 sim_fast_bits only (p == P, m >= P); a restart whose simulation
+// saturates is abandoned and its id appended to A.redo.  FAST = false: the exact int64
+// sim_exact (runtime p <= P), over [r_lo, r_hi) or over the ids listed in A.redo.
+template <int P, bool FAST>
 __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
@@ -692,10 +797,18 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
     return diff;
   };
 
+  unsigned int rsims = 0;  // simulations of the current restart
   for (;;) {
     if (phase == 0) {
-      r = atomicAdd(A.counter, 1u) + A.r_lo;
-      if (r >= A.r_hi) break;
+      if (!FAST && A.redo) {
+        const unsigned int i = atomicAdd(A.counter, 1u);
+        if (i >= A.redo[0]) break;
+        r = A.redo[1 + i];
+      } else {
+        r = atomicAdd(A.counter, 1u) + A.r_lo;
+        if (r >= A.r_hi) break;
+      }
+      rsims = 0;
       // restart start: Alg. 1 (r = 0) or the seeded perturbation (reading Q21)
       cand[0] = 0;
 #pragma unroll
@@ -721,10 +834,30 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
     int64_t F[P], B[P], C[P];
     stage_costs<P>(T, p, cc, F, B, C);
     uint32_t pb[P];
-    const int64_t Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
+#pragma unroll
+    for (int x = 0; x < P; ++x) pb[x] = 0;
+    int64_t Tc;
+    if constexpr (FAST) {
+      uint32_t wF[P], wB[P];
+#pragma unroll
+      for (int x = 0; x < P; ++x) {
+        wF[x] = (uint32_t)(F[x] + ((x > 0) ? C[x - 1] : 0));
+        wB[x] = (uint32_t)(B[x] + C[x]);
+      }
+      const uint32_t t32 = sim_fast_bits<P>(m, wF, wB, A.S, A.CR, br);
+      if (t32 >= A.S) {  // not exact: hand the whole restart to the int64 pass
+        const unsigned int slot = atomicAdd(&A.redo[0], 1u);
+        A.redo[1 + slot] = r;
+        phase = 0;
+        continue;
+      }
+      Tc = (int64_t)t32;
+    } else {
+      Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
+    }
     int len;
     const int Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
-    ++nsims;
+    ++rsims;
     bool do_step = false, finish = false;
     if (phase == 1) {
       curM = Mc;
@@ -778,9 +911,13 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
       }
     }
     if (finish) {
+      nsims += rsims;
       if (bestT < (1ll << 43)) lane_key = min(lane_key, ((unsigned long long)bestT << 20) | r);
       if (A.replay)
         for (int x = 1; x <= p - 1; ++x) A.replay[x - 1] = best[x];
+      if (A.best_out)
+        for (int x = 1; x <= p - 1; ++x)
+          A.best_out[(size_t)(r - A.r_lo) * (p - 1) + (x - 1)] = (int16_t)best[x];
       phase = 0;
     }
   }
@@ -1080,8 +1217,8 @@ cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, u
   }
 }
 
-template <int P>
-static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev) {
+template <int P, bool FAST>
+static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev, uint64_t nwork) {
   const int threads = A.replay ? 32 : 128;
   const int rows = A.m + min(A.p - 1, A.m);
   const size_t narg = (size_t)(A.t.n + 1) * (A.p + 1);
@@ -1089,18 +1226,17 @@ static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev) {
                       ((narg + 7) & ~size_t(7)) * 2 + 32 * 4;
   const size_t smem = base + (size_t)rows * BitsLayout<P>::WPR * 4 * threads;
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
-  cudaError_t e = set_smem((const void*)k_heur<P>, smem);
+  cudaError_t e = set_smem((const void*)k_heur<P, FAST>, smem);
   if (e != cudaSuccess) return e;
   int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_heur<P>, threads, smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_heur<P, FAST>, threads, smem);
   if (e != cudaSuccess) return e;
   occ = occ < 1 ? 1 : occ;
-  const uint64_t R = A.r_hi - A.r_lo;
   uint64_t blocks = (uint64_t)num_sms(dev) * occ;
-  const uint64_t need = (R + threads - 1) / threads;
+  const uint64_t need = (nwork + threads - 1) / threads;
   if (blocks > need) blocks = need;
   if (blocks < 1) blocks = 1;
-  k_heur<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+  k_heur<P, FAST><<<(unsigned)blocks, threads, smem, s>>>(A);
   return cudaGetLastError();
 }
 
@@ -1108,16 +1244,42 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
                              uint32_t r_lo, uint32_t r_hi, const int16_t* arg,
                              const int32_t* alg1_cuts, unsigned int* counter,
                              unsigned long long* key, int32_t* replay_cuts,
-                             unsigned long long* sims, cudaStream_t s) {
+                             unsigned long long* sims, int16_t* best_out, uint32_t fastS,
+                             int fastCR, cudaStream_t s) {
   int dev = 0;
   cudaGetDevice(&dev);
-  HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts, sims};
-  switch (pick_P(p)) {
-    case 2: return heur_P<2>(A, s, dev);
-    case 4: return heur_P<4>(A, s, dev);
-    case 8: return heur_P<8>(A, s, dev);
-    case 16: return heur_P<16>(A, s, dev);
-    default: return heur_P<32>(A, s, dev);
+  // counter[0]: restart cursor of the first pass; counter[1]: cursor of the redo
+  // pass; counter[2]: redo count; counter[3..]: redo ids (caller zeroes [0..2])
+  const bool fast = fastS > 0 && pick_P(p) == p && p >= 2 && p <= 16 && m >= p && !replay_cuts;
+  HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts, sims,
+             best_out, fastS, fastCR < 1 ? 1 : fastCR, nullptr};
+  const uint64_t R = r_hi - r_lo;
+  if (!fast) {
+    switch (pick_P(p)) {
+      case 2: return heur_P<2, false>(A, s, dev, R);
+      case 4: return heur_P<4, false>(A, s, dev, R);
+      case 8: return heur_P<8, false>(A, s, dev, R);
+      case 16: return heur_P<16, false>(A, s, dev, R);
+      default: return heur_P<32, false>(A, s, dev, R);
+    }
+  }
+  A.redo = counter + 2;
+  cudaError_t e;
+  switch (p) {
+    case 2: e = heur_P<2, true>(A, s, dev, R); break;
+    case 4: e = heur_P<4, true>(A, s, dev, R); break;
+    case 8: e = heur_P<8, true>(A, s, dev, R); break;
+    default: e = heur_P<16, true>(A, s, dev, R); break;
+  }
+  if (e != cudaSuccess) return e;
+  // exact pass over the abandoned restarts (exits at once when the list is empty)
+  HeurArgs B = A;
+  B.counter = counter + 1;
+  switch (p) {
+    case 2: return heur_P<2, false>(B, s, dev, 128);
+    case 4: return heur_P<4, false>(B, s, dev, 128);
+    case 8: return heur_P<8, false>(B, s, dev, 128);
+    default: return heur_P<16, false>(B, s, dev, 128);
   }
 }
 
@@ -1177,7 +1339,7 @@ cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t*
 cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s) {
   k_init_key<<<1, 1, 0, s>>>(key);
   if (counter) {
-    cudaError_t e = cudaMemsetAsync(counter, 0, sizeof(unsigned int), s);
+    cudaError_t e = cudaMemsetAsync(counter, 0, 3 * sizeof(unsigned int), s);  // cursors + redo count
     if (e != cudaSuccess) return e;
   }
   return cudaGetLastError();

@@ -41,12 +41,15 @@ cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, u
                          SweepPlan* plan_out);
 
 // Heuristic restarts [r_lo, r_hi); key = min (T << 20 | r).  replay_cuts (int32[p-1])
-// non-null: single-restart replay writing that restart's best cut vector.
+// non-null: single-restart replay writing that restart's best cut vector.  counter
+// must hold 3 + (r_hi - r_lo) words (cursors, redo count, redo ids).  fastS > 0 enables
+// the u32 pass (restarts that saturate are redone by an exact int64 pass).
 cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, int radius,
                              uint32_t r_lo, uint32_t r_hi, const int16_t* arg,
                              const int32_t* alg1_cuts, unsigned int* counter,
                              unsigned long long* key, int32_t* replay_cuts,
-                             unsigned long long* sims, cudaStream_t s);
+                             unsigned long long* sims, int16_t* best_out, uint32_t fastS,
+                             int fastCR, cudaStream_t s);
 
 struct OpRec {
   int32_t stage, kind, microbatch, piece;
@@ -59,7 +62,7 @@ cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t*
                          int cap, int32_t* len_master, int64_t* T, void* scratch,
                          cudaStream_t s);
 
-// key = INT64_MAX (and *counter = 0 if non-null); precedes launch_sweep/heuristic.
+// key = INT64_MAX (and counter[0..2] = 0 if non-null); precedes launch_sweep/heuristic.
 cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s);
 
 // Decode helper: unrank lex rank -> cut vector int32[p-1].

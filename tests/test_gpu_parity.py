@@ -442,3 +442,29 @@ def test_search_modes_equal_configs(ap, cfg):
         for lo in (0, N // 3, N - 5000):
             ks = [_search_mode(ap, plan, wl.p, wl.m, 1, 8, mode, lo, lo + 5000) for mode in (0, 1, 2)]
             assert ks[0] == ks[1] == ks[2]
+
+
+@pytest.mark.parametrize("mode", ["", "int64", "redo"])
+def test_heuristic_fast_and_redo_paths(ap, oracle_mod, monkeypatch, mode):
+    """The u32 restart kernel, the exact int64 kernel, and the u32 kernel with a bound
+    so low that many restarts saturate and are redone exactly, all give the oracle's
+    winner and simulation count (C2, p=4: the fast path applies)."""
+    import torch
+    wl = synth.config(2)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model.from_workload(wl)
+    R = 1024
+    o = M.heuristic(wl.p, wl.m, wl.seed, wl.radius, 0, R, per_restart=True)
+    if mode == "int64":
+        monkeypatch.setenv("AP_HEUR", "int64")
+    if mode == "redo":
+        monkeypatch.setenv("AP_HEUR_S", str(int(np.median(o["per_restart_T"]))))
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, R, 0, key)
+    torch.cuda.synchronize()
+    kv = int(key.item())
+    assert (kv >> 20, kv & 0xFFFFF) == (o["T"], o["restart"])
+    assert ap.ap_last_sims() == o["sims"]
+    res = ap.ap_decode(plan, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=kv)
+    assert res["cuts"] == [int(x) for x in o["cuts"]]

@@ -1,0 +1,18 @@
+"""One C5 heuristic plan (65 536 restarts + decode + Slicer sweep), for profiling."""
+import os, sys, time
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch
+import synth
+import paper_conf_cluster_liulldgl22_b200 as ap
+wl = synth.config(5)
+f, b, a = wl.arrays()
+plan = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s)
+key = torch.empty(1, dtype=torch.int64, device="cuda")
+for rep in range(int(sys.argv[1]) if len(sys.argv) > 1 else 3):
+    torch.cuda.synchronize(); t0 = time.perf_counter()
+    ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, wl.restarts, 0, key)
+    kv = int(key.item()); t1 = time.perf_counter()
+    kms = ap.ap_last_kernel_ms(); sims = ap.ap_last_sims()
+    res = ap.ap_decode(plan, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=kv); t2 = time.perf_counter()
+    T, bk = ap.ap_slice_sweep(plan, wl.p, wl.m, res["cuts"], 16); t3 = time.perf_counter()
+    print(f"search {1e3*(t1-t0):.2f} ms (kernel {kms:.2f} ms, {sims} sims, {sims/kms*1e3:.3e} sims/s) decode {1e3*(t2-t1):.2f} ms slice {1e3*(t3-t2):.2f} ms T {res['time_ns']} r {res['restart']}", flush=True)

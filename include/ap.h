@@ -164,7 +164,7 @@ ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, i
 
 /*
  * ap_search_heuristic -- AutoPipe's boundary-shifting heuristic (PAPER.md:147-198,
- * steps 1, 3, 4; step 2 / Eq. (1) is adjust_mode 1, not yet supported), run as
+ * steps 1, 3, 4; adjust_mode 1 adds step 2 / Eq. (1)), run as
  * independent deterministic restarts r in [r_lo, r_hi), one GPU lane each.
  * Restart 0 starts at the Algorithm 1 partition; restart r >= 1 at
  * the seeded perturbation of DESIGN.md reading Q21 (splitmix64(seed ^ r<<32 ^ x),
@@ -175,7 +175,12 @@ ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, i
  * child with master <= i and least (T, child order); stop if none.  A restart's
  * result is the first-visited partition of least T among all it simulated.  k = 1.
  *   key   device int64[1]: min over restarts of (T << 20 | r), INT64_MAX if none.
- *   0 <= r_lo < r_hi <= 2^20, 0 <= radius <= 1<<20, adjust_mode must be 0.
+ *   adjust_mode 1 (reading Q19/Q20): before each step, for s = i+1..p-2 while
+ *   sum_{j=i+1..s}(F_j+B_j) > (s-i)*B_i and stage s has >= 2 blocks, move its last
+ *   block to s+1 and re-simulate; stop adjusting when the master changes.  Because the
+ *   master can then rise, the walk also stops when its post-adjustment scheme repeats
+ *   one of its last 32 (splitmix64 hash of the cut vector); the n*p step cap holds.
+ *   0 <= r_lo < r_hi <= 2^20, 0 <= radius <= 1<<20, adjust_mode in {0, 1}.
  * Synchronises `stream` once (overflow guard), then launches asynchronously.
  */
 ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,

@@ -86,6 +86,12 @@ def _load():
             lib.or_heuristic.restype = i32
             lib.or_heuristic.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64, i32, u32,
                                          u32, P(i64), P(u32), P(i32), P(i64), P(u64)]
+            lib.or_heuristic_ex.restype = i32
+            lib.or_heuristic_ex.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64, i32, u32,
+                                            u32, i32, P(i64), P(u32), P(i32), P(i64), P(u64)]
+            lib.or_heuristic_restart_ex.restype = i32
+            lib.or_heuristic_restart_ex.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64,
+                                                    i32, u32, i32, P(i64), P(i32), P(u64), P(i32)]
             lib.or_slice_sweep.restype = i32
             lib.or_slice_sweep.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, P(i32), i32,
                                            P(i64), P(i32)]
@@ -235,40 +241,41 @@ class Model:
         lib.or_restart_start(self.n, p, _p(a1, C.c_int32), seed, radius, r, _p(out, C.c_int32))
         return out[: p - 1].copy()
 
-    def heuristic_restart(self, p, m, seed, radius, r):
+    def heuristic_restart(self, p, m, seed, radius, r, adjust_mode: int = 0):
         lib = _load()
         T = C.c_int64(); sims = C.c_uint64(); steps = C.c_int32()
         cuts = np.zeros(max(p - 1, 1), np.int32)
-        _chk(lib.or_heuristic_restart(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
-                                      _p(self.comm, C.c_int64), p, m, seed, radius, r,
-                                      C.byref(T), _p(cuts, C.c_int32), C.byref(sims),
-                                      C.byref(steps)))
+        _chk(lib.or_heuristic_restart_ex(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                                         _p(self.comm, C.c_int64), p, m, seed, radius, r,
+                                         adjust_mode, C.byref(T), _p(cuts, C.c_int32),
+                                         C.byref(sims), C.byref(steps)))
         return {"T": T.value, "cuts": cuts[: p - 1].copy(), "sims": sims.value,
                 "steps": steps.value}
 
-    def heuristic(self, p, m, seed, radius, r_lo, r_hi, per_restart: bool = False):
+    def heuristic(self, p, m, seed, radius, r_lo, r_hi, per_restart: bool = False,
+                  adjust_mode: int = 0):
         lib = _load()
         T = C.c_int64(); r = C.c_uint32(); sims = C.c_uint64()
         cuts = np.zeros(max(p - 1, 1), np.int32)
         per = np.zeros(max(r_hi - r_lo, 1), np.int64)
-        _chk(lib.or_heuristic(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
-                              _p(self.comm, C.c_int64), p, m, seed, radius, r_lo, r_hi,
-                              C.byref(T), C.byref(r), _p(cuts, C.c_int32), _p(per, C.c_int64),
-                              C.byref(sims)))
+        _chk(lib.or_heuristic_ex(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                                 _p(self.comm, C.c_int64), p, m, seed, radius, r_lo, r_hi,
+                                 adjust_mode, C.byref(T), C.byref(r), _p(cuts, C.c_int32),
+                                 _p(per, C.c_int64), C.byref(sims)))
         out = {"T": T.value, "restart": r.value, "cuts": cuts[: p - 1].copy(), "sims": sims.value}
         if per_restart:
             out["per_restart_T"] = per[: r_hi - r_lo].copy()
         return out
 
     def heuristic_parallel(self, p, m, seed, radius, r_lo, r_hi, threads=None,
-                           per_restart: bool = False):
+                           per_restart: bool = False, adjust_mode: int = 0):
         threads = threads or os.cpu_count() or 1
         tot = r_hi - r_lo
         edges = [r_lo + (tot * i) // threads for i in range(threads + 1)]
         idx = [i for i in range(threads) if edges[i + 1] > edges[i]]
         with ThreadPoolExecutor(threads) as ex:
             res = list(ex.map(lambda i: self.heuristic(p, m, seed, radius, edges[i], edges[i + 1],
-                                                       per_restart), idx))
+                                                       per_restart, adjust_mode), idx))
         best = dict(min(res, key=lambda d: (d["T"], d["restart"])))
         best["sims"] = sum(d["sims"] for d in res)
         if per_restart:

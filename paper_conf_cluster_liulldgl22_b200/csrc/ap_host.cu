@@ -65,7 +65,7 @@ thread_local KernelTimer g_timer;
 // ap_decode(mode 1) can read the winner's cuts instead of replaying its walk.
 struct HeurCache {
   uint64_t plan_gen = 0;
-  int p = 0, m = 0, radius = 0, dev = -1;
+  int p = 0, m = 0, radius = 0, dev = -1, adjust_mode = 0;
   uint64_t seed = 0;
   uint32_t r_lo = 0, r_hi = 0;
   int16_t* d_best = nullptr;
@@ -561,7 +561,8 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   ap_status st = check_pm(plan, p, m);
   if (st != AP_OK) return st;
   if (!key) return fail(AP_ERR_INVALID, "key is NULL");
-  if (adjust_mode != 0) return fail(AP_ERR_INVALID, "adjust_mode %d not supported (only 0)", adjust_mode);
+  if (adjust_mode != 0 && adjust_mode != 1)
+    return fail(AP_ERR_INVALID, "adjust_mode %d (0 none, 1 Eq. (1))", adjust_mode);
   if (r_lo >= r_hi || r_hi > (1u << 20)) return fail(AP_ERR_INVALID, "restart range [%u, %u)", r_lo, r_hi);
   if (radius < 0 || radius > (1 << 20)) return fail(AP_ERR_INVALID, "radius %d", radius);
   cudaStream_t s = S_(stream);
@@ -611,7 +612,7 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_heuristic(plan->dev(), p, m, seed, radius, r_lo, r_hi, d_arg, d_a1, d_ctr,
                                 reinterpret_cast<unsigned long long*>(key), nullptr, d_sims,
-                                g_hcache.d_best, fastS, hCR, s));
+                                g_hcache.d_best, fastS, hCR, adjust_mode, s));
   g_hcache.plan_gen = plan->gen;
   g_hcache.p = p;
   g_hcache.m = m;
@@ -619,6 +620,7 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   g_hcache.radius = radius;
   g_hcache.r_lo = r_lo;
   g_hcache.r_hi = r_hi;
+  g_hcache.adjust_mode = adjust_mode;
   g_hcache.valid = true;
   AP_CUDA(g_timer.record(1, s, plan->device));
   g_timer.sims_on_device = true;
@@ -675,7 +677,8 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
         }
       }
     } else if (res == AP_OK && mode == 1) {
-      if (adjust_mode != 0) res = fail(AP_ERR_INVALID, "adjust_mode %d", adjust_mode);
+      if (adjust_mode != 0 && adjust_mode != 1)
+        res = fail(AP_ERR_INVALID, "adjust_mode %d", adjust_mode);
       keyT = key >> 20;
       const uint32_t r = (uint32_t)(key & ((1 << 20) - 1));
       out->restart = r;
@@ -687,6 +690,7 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
       unsigned int* d_ctr;
       unsigned long long* d_key;
       const bool cached = g_hcache.valid && g_hcache.plan_gen == plan->gen && g_hcache.p == p &&
+                          g_hcache.adjust_mode == adjust_mode &&
                           g_hcache.m == m && g_hcache.seed == seed &&
                           g_hcache.radius == radius && r >= g_hcache.r_lo &&
                           r < g_hcache.r_hi && g_hcache.dev == plan->device && p > 1;
@@ -709,7 +713,7 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
         if (e == cudaSuccess) e = apk::launch_init_key(d_key, d_ctr, s);
         if (e == cudaSuccess)
           e = apk::launch_heuristic(plan->dev(), p, m, seed, radius, r, r + 1, d_arg, d_a1, d_ctr,
-                                    d_key, d_cuts, nullptr, nullptr, 0, 1, s);
+                                    d_key, d_cuts, nullptr, nullptr, 0, 1, adjust_mode, s);
         if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "replay: %s", cudaGetErrorString(e));
       }
     } else if (res == AP_OK) {

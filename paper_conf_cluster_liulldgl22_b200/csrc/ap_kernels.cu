@@ -733,6 +733,7 @@ struct HeurArgs {
   int CR;                    // fast path: rows between clamps
   unsigned int* redo;        // FAST: [0] = count, [1..] restarts abandoned on saturation;
                              // generic: if non-null, run exactly the listed restarts
+  int adjust_mode;           // 0 none, 1 Eq. (1) step 2
 };
 
 // Algorithm 1 on the prefix [0, c) with j stages: writes c_1..c_{j-1} (line 15).
@@ -797,6 +798,64 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
     return diff;
   };
 
+  // ---- paper step 2 (adjust_mode 1): Eq. (1), reading Q19/Q20, DESIGN.md §2
+  int adj_i = 0, adj_s = 0, nring = 0;
+  uint64_t ring[32];
+  // first s >= adj_s (<= p-2) where Eq. (1) is violated for master adj_i and stage s
+  // still has >= 2 blocks; on success cand = cur with stage s's last block moved to s+1
+  auto adj_find = [&]() -> bool {
+    for (; adj_s <= p - 2; ++adj_s) {
+      const int i = adj_i;
+      const int64_t lhs = (T.Pf[cur[adj_s + 1]] + T.Pb[cur[adj_s + 1]]) -
+                          (T.Pf[cur[i + 1]] + T.Pb[cur[i + 1]]);
+      const int64_t Bi = T.Pb[cur[i + 1]] - T.Pb[cur[i]];
+      if (lhs > (int64_t)(adj_s - i) * Bi && cur[adj_s + 1] - cur[adj_s] >= 2) {
+#pragma unroll
+        for (int x = 0; x <= P; ++x) cand[x] = cur[x];
+        cand[adj_s + 1] -= 1;
+        phase = 3;
+        return true;
+      }
+    }
+    return false;
+  };
+  auto start_children = [&]() -> bool {
+    ++steps;
+    selT = INT64_MAX;
+    for (int idx = 0; idx <= 3; ++idx)
+      if (gen_child(idx, curM)) {
+        chIdx = idx;
+        phase = 2;
+        return true;
+      }
+    return false;
+  };
+  // after the adjustment: stop on a repeated scheme (mode 1), stop at master 0,
+  // otherwise generate the children of step 3
+  auto post_adjust = [&]() -> bool {
+    if (A.adjust_mode == 1) {
+      uint64_t h = 0;
+      for (int x = 1; x <= p - 1; ++x) h = splitmix64(h ^ (uint64_t)(uint32_t)cur[x]);
+      bool seen = false;
+      for (int q = 0; q < nring && q < 32; ++q) seen = seen || (ring[q] == h);
+      if (seen) return false;
+      ring[nring % 32] = h;
+      ++nring;
+    }
+    if (curM == 0) return false;
+    return start_children();
+  };
+  // top of a walk step: the step cap, then (mode 1) the Eq. (1) adjustment
+  auto begin_step = [&]() -> bool {
+    if (steps >= smax) return false;
+    if (A.adjust_mode == 1 && p >= 3) {
+      adj_i = curM;
+      adj_s = curM + 1;
+      if (adj_find()) return true;
+    }
+    return post_adjust();
+  };
+
   unsigned int rsims = 0;  // simulations of the current restart
   for (;;) {
     if (phase == 0) {
@@ -858,7 +917,7 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
     int len;
     const int Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
     ++rsims;
-    bool do_step = false, finish = false;
+    bool ready;  // true: the next candidate is in cand; false: the restart is finished
     if (phase == 1) {
       curM = Mc;
       bestT = Tc;
@@ -867,8 +926,9 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
         best[x] = cand[x];
       }
       steps = 0;
-      do_step = true;
-    } else {
+      nring = 0;
+      ready = begin_step();
+    } else if (phase == 2) {
       if (Tc < bestT) {
         bestT = Tc;
         for (int x = 0; x <= p; ++x) best[x] = cand[x];
@@ -884,32 +944,31 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
           chIdx = idx;
           found = true;
         }
-      if (!found) {
-        if (selT == INT64_MAX) {
-          finish = true;
-        } else {
-          for (int x = 0; x <= p; ++x) cur[x] = sel[x];
-          curM = selM;
-          do_step = true;
-        }
-      }
-    }
-    if (do_step) {
-      if (curM == 0 || steps >= smax) {
-        finish = true;
+      if (found) {
+        ready = true;
+      } else if (selT == INT64_MAX) {
+        ready = false;  // no child qualifies
       } else {
-        ++steps;
-        selT = INT64_MAX;
-        bool found = false;
-        for (int idx = 0; idx <= 3 && !found; ++idx)
-          if (gen_child(idx, curM)) {
-            chIdx = idx;
-            found = true;
-          }
-        if (!found) finish = true;
-        else phase = 2;
+        for (int x = 0; x <= p; ++x) cur[x] = sel[x];
+        curM = selM;
+        ready = begin_step();
+      }
+    } else {  // phase 3: an Eq. (1) adjustment was simulated
+      if (Tc < bestT) {
+        bestT = Tc;
+        for (int x = 0; x <= p; ++x) best[x] = cand[x];
+      }
+      for (int x = 0; x <= p; ++x) cur[x] = cand[x];
+      if (Mc != adj_i) {
+        curM = Mc;  // "if the master stage changes ..., stop the adjustment"
+        ready = post_adjust();
+      } else if (adj_find()) {
+        ready = true;
+      } else {
+        ready = post_adjust();
       }
     }
+    const bool finish = !ready;
     if (finish) {
       nsims += rsims;
       if (bestT < (1ll << 43)) lane_key = min(lane_key, ((unsigned long long)bestT << 20) | r);
@@ -1245,14 +1304,14 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
                              const int32_t* alg1_cuts, unsigned int* counter,
                              unsigned long long* key, int32_t* replay_cuts,
                              unsigned long long* sims, int16_t* best_out, uint32_t fastS,
-                             int fastCR, cudaStream_t s) {
+                             int fastCR, int adjust_mode, cudaStream_t s) {
   int dev = 0;
   cudaGetDevice(&dev);
   // counter[0]: restart cursor of the first pass; counter[1]: cursor of the redo
   // pass; counter[2]: redo count; counter[3..]: redo ids (caller zeroes [0..2])
   const bool fast = fastS > 0 && pick_P(p) == p && p >= 2 && p <= 16 && m >= p && !replay_cuts;
   HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts, sims,
-             best_out, fastS, fastCR < 1 ? 1 : fastCR, nullptr};
+             best_out, fastS, fastCR < 1 ? 1 : fastCR, nullptr, adjust_mode};
   const uint64_t R = r_hi - r_lo;
   if (!fast) {
     switch (pick_P(p)) {

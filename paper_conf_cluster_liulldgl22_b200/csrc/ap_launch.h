@@ -49,7 +49,7 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
                              const int32_t* alg1_cuts, unsigned int* counter,
                              unsigned long long* key, int32_t* replay_cuts,
                              unsigned long long* sims, int16_t* best_out, uint32_t fastS,
-                             int fastCR, cudaStream_t s);
+                             int fastCR, int adjust_mode, cudaStream_t s);
 
 struct OpRec {
   int32_t stage, kind, microbatch, piece;

@@ -468,3 +468,44 @@ def test_heuristic_fast_and_redo_paths(ap, oracle_mod, monkeypatch, mode):
     assert ap.ap_last_sims() == o["sims"]
     res = ap.ap_decode(plan, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=kv)
     assert res["cuts"] == [int(x) for x in o["cuts"]]
+
+
+@pytest.mark.parametrize("cfg,R", [(2, 512), (3, 256), (5, 1024)])
+def test_heuristic_adjust_eq1_vs_oracle(ap, oracle_mod, cfg, R):
+    """adjust_mode 1 (paper step 2, Eq. (1)): GPU winner, decode and simulation count
+    equal the oracle's walk with the same reading (Q19)."""
+    import torch
+    wl = synth.config(cfg)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model.from_workload(wl)
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, R, 1, key)
+    torch.cuda.synchronize()
+    kv = int(key.item())
+    o = M.heuristic_parallel(wl.p, wl.m, wl.seed, wl.radius, 0, R, adjust_mode=1)
+    assert (kv >> 20, kv & 0xFFFFF) == (o["T"], o["restart"])
+    assert ap.ap_last_sims() == o["sims"]
+    res = ap.ap_decode(plan, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, adjust_mode=1, key=kv)
+    assert res["cuts"] == [int(x) for x in o["cuts"]]
+
+
+def test_heuristic_adjust_eq1_random(ap, oracle_mod):
+    import torch
+    rng = np.random.default_rng(77)
+    for trial in range(8):
+        n = int(rng.integers(8, 30))
+        f, b, a = synth.random_tables(trial + 50, n, ["b3f", "uniform"][trial % 2])
+        M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+        plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+        p = int(rng.choice([3, 4, 5, 8]))
+        if p > n:
+            continue
+        m = int(rng.integers(1, 3 * p))
+        key = torch.empty(1, dtype=torch.int64, device="cuda")
+        ap.ap_search_heuristic(plan, p, m, 0x5EED, 2, 0, 200, 1, key)
+        torch.cuda.synchronize()
+        kv = int(key.item())
+        o = M.heuristic(p, m, 0x5EED, 2, 0, 200, adjust_mode=1)
+        assert (kv >> 20, kv & 0xFFFFF) == (o["T"], o["restart"]), (n, p, m)
+        assert ap.ap_last_sims() == o["sims"]

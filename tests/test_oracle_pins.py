@@ -608,3 +608,23 @@ def test_kfactor_identity_on_oracle_dag(oracle_mod):
                 G_ref = G
             assert G == G_ref
             assert max(FF[x] + G[x] for x in range(p)) == r["T"]
+
+
+def test_heuristic_eq1_properties(oracle_mod):
+    """adjust_mode 1: opt <= result <= T(start), deterministic, bounded walk; mode 0
+    unchanged by the mode-1 machinery (P13 for step 2)."""
+    for seed in range(20):
+        n = 8 + seed % 10
+        f, b, a = synth.random_tables(seed, n, "b3f")
+        M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+        p = 3 + seed % 3
+        m = p + 2 * (seed % 3)
+        opt = M.exhaustive(p, m)["T"]
+        for r in range(3):
+            st = M.restart_start(p, 0x5EED, 2, r)
+            h1 = M.heuristic_restart(p, m, 0x5EED, 2, r, adjust_mode=1)
+            assert opt <= h1["T"] <= M.T(p, m, st)
+            assert M.T(p, m, h1["cuts"]) == h1["T"]
+            h2 = M.heuristic_restart(p, m, 0x5EED, 2, r, adjust_mode=1)
+            assert (h2["T"], list(h2["cuts"]), h2["sims"]) == (h1["T"], list(h1["cuts"]), h1["sims"])
+            assert h1["steps"] <= n * p

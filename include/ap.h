@@ -219,6 +219,27 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
 ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
                          int32_t k_max, int64_t* time_ns, int32_t* best_k);
 
+/*
+ * ap_slice_sweep_paper -- the paper's own Slicer form (Fig. 8): the
+ * forwards of the first s micro-batches are split into k pieces each (k = 2: halves)
+ * and BP is never sliced.  T(s) for s = 0..s_max (s = 0: no slicing); best_s =
+ * argmin (T, s).  T only (no critical path for s > 1).  Blocking.
+ *   cuts host int32[p-1]; time_ns host int64[s_max+1]; 0 <= s_max <= m.
+ */
+ap_status ap_slice_sweep_paper(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                               int32_t k, int32_t s_max, int64_t* time_ns, int32_t* best_s);
+
+/*
+ * ap_slicer_alg2 -- Algorithm 2, the Slicer's analytic number mb of
+ * leading micro-batches to slice in halves, transcribed on the device.  The printed
+ * pseudocode is garbled; readings in DESIGN.md §2 (Q22-Q24).  reading 0 = the
+ * pseudocode's stop test (line 34, "tempt <= endt[0][1]"), reading 1 = the text's
+ * ("start of the unbroken micro-batch >= end of the second half").
+ * Blocking.  cuts host int32[p-1]; *mb in [1, p].
+ */
+ap_status ap_slicer_alg2(const ap_plan* plan, int32_t p, const int32_t* cuts, int32_t reading,
+                         int32_t* mb);
+
 typedef struct {
   int32_t stage;       /* x                                        */
   int32_t kind;        /* 0 = forward (FP), 1 = backward (BP)      */

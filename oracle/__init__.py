@@ -92,6 +92,11 @@ def _load():
             lib.or_heuristic_restart_ex.restype = i32
             lib.or_heuristic_restart_ex.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64,
                                                     i32, u32, i32, P(i64), P(i32), P(u64), P(i32)]
+            lib.or_slice_sweep_paper.restype = i32
+            lib.or_slice_sweep_paper.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, P(i32),
+                                                 i32, i32, P(i64), P(i32)]
+            lib.or_alg2.restype = i32
+            lib.or_alg2.argtypes = [i32, P(i64), P(i64), P(i64), i32, P(i32), i32, P(i32)]
             lib.or_slice_sweep.restype = i32
             lib.or_slice_sweep.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, P(i32), i32,
                                            P(i64), P(i32)]
@@ -290,6 +295,29 @@ class Model:
                                 _p(self.comm, C.c_int64), p, m, _p(c, C.c_int32), K,
                                 _p(T, C.c_int64), C.byref(bk)))
         return T, bk.value
+
+
+def _slice_paper(self, p, m, cuts, k, s_max):
+    lib = _load()
+    c = _i32(cuts) if p > 1 else np.zeros(1, np.int32)
+    T = np.zeros(s_max + 1, np.int64); bs = C.c_int32()
+    _chk(lib.or_slice_sweep_paper(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                                  _p(self.comm, C.c_int64), p, m, _p(c, C.c_int32), k, s_max,
+                                  _p(T, C.c_int64), C.byref(bs)))
+    return T, bs.value
+
+
+def _alg2(self, p, cuts, reading=0):
+    lib = _load()
+    c = _i32(cuts) if p > 1 else np.zeros(1, np.int32)
+    mb = C.c_int32()
+    _chk(lib.or_alg2(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                     _p(self.comm, C.c_int64), p, _p(c, C.c_int32), reading, C.byref(mb)))
+    return mb.value
+
+
+Model.slice_sweep_paper = _slice_paper
+Model.alg2 = _alg2
 
 
 def count(n: int, p: int) -> int:

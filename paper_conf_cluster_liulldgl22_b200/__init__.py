@@ -80,6 +80,10 @@ def _load_lib():
     lib.ap_decode.argtypes = [vp, i32, i32, i32, i32, i32, u64, i32, i32, i64, P(ApResult)]
     lib.ap_slice_sweep.restype = i32
     lib.ap_slice_sweep.argtypes = [vp, i32, i32, P(i32), i32, P(i64), P(i32)]
+    lib.ap_slice_sweep_paper.restype = i32
+    lib.ap_slice_sweep_paper.argtypes = [vp, i32, i32, P(i32), i32, i32, P(i64), P(i32)]
+    lib.ap_slicer_alg2.restype = i32
+    lib.ap_slicer_alg2.argtypes = [vp, i32, P(i32), i32, P(i32)]
     lib.ap_critical_path.restype = i32
     lib.ap_critical_path.argtypes = [vp, i32, i32, i32, P(i32), P(ApOp), i32, P(i32), P(i32),
                                      P(i64)]
@@ -100,7 +104,8 @@ lib = _load_lib()
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
            "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_exhaustive_mode",
            "ap_search_heuristic",
-           "ap_decode", "ap_slice_sweep", "ap_critical_path", "ap_alg1", "ap_last_launch",
+           "ap_decode", "ap_slice_sweep", "ap_slice_sweep_paper", "ap_slicer_alg2",
+           "ap_critical_path", "ap_alg1", "ap_last_launch",
            "ap_last_kernel_ms", "ap_last_sims")
 
 
@@ -255,6 +260,26 @@ def ap_slice_sweep(plan: Plan, p: int, m: int, cuts: Sequence[int], k_max: int):
     _check(lib.ap_slice_sweep(plan.handle, int(p), int(m), c.ctypes.data_as(C.POINTER(C.c_int32)),
                               int(k_max), T.ctypes.data_as(C.POINTER(C.c_int64)), C.byref(bk)))
     return T, bk.value
+
+
+def ap_slice_sweep_paper(plan: Plan, p: int, m: int, cuts: Sequence[int], k: int, s_max: int):
+    """T(s) for s = 0..s_max with the first s micro-batches' forwards in k pieces."""
+    c = _i32(cuts) if p > 1 else np.zeros(1, np.int32)
+    T = np.zeros(int(s_max) + 1, np.int64)
+    bs = C.c_int32()
+    _check(lib.ap_slice_sweep_paper(plan.handle, int(p), int(m),
+                                    c.ctypes.data_as(C.POINTER(C.c_int32)), int(k), int(s_max),
+                                    T.ctypes.data_as(C.POINTER(C.c_int64)), C.byref(bs)))
+    return T, bs.value
+
+
+def ap_slicer_alg2(plan: Plan, p: int, cuts: Sequence[int], reading: int = 1) -> int:
+    """Algorithm 2's mb (reading 0: pseudocode stop test, 1: the text's)."""
+    c = _i32(cuts) if p > 1 else np.zeros(1, np.int32)
+    mb = C.c_int32()
+    _check(lib.ap_slicer_alg2(plan.handle, int(p), c.ctypes.data_as(C.POINTER(C.c_int32)),
+                              int(reading), C.byref(mb)))
+    return mb.value
 
 
 def ap_critical_path(plan: Plan, p: int, m: int, k: int, cuts: Sequence[int],

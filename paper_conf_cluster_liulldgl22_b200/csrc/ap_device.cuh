@@ -281,6 +281,119 @@ AP_DEV_INLINE int64_t sim_exact(int p, int m, int k, const int64_t (&F)[P],
   return L[0];
 }
 
+// The paper's Slicer form: micro-batches 0..s-1 have their
+// forward split into k pieces (s = 0: none).  Same row sweep as sim_exact (MODE 0,
+// T only).  A sliced F(x, j, q) depends on F(x-1, j, q) and on the stage's previous
+// op (piece q-1, or for q = 0 the stage's last op L[x]).  PV[x][.] holds the pieces
+// of stage x's latest sliced forward; because the forward pass runs x ascending and
+// stage x-1 may already have sliced F(x-1, j+1) in this row (w_{x-1} = w_x + 1),
+// the cross pieces are taken from a copy saved before that overwrite.
+template <int P>
+AP_DEV_INLINE int64_t sim_sliced(int p, int m, int s, int k, const int64_t (&F)[P],
+                                 const int64_t (&B)[P], const int64_t (&C)[P]) {
+  if (s <= 0) k = 1;
+  if (k <= 1) s = 0;
+  int64_t wF[P], wB[P], FF[P], L[P];
+  int w[P];
+  int64_t PV[P][kMaxK];
+#pragma unroll
+  for (int x = 0; x < P; ++x) {
+    wF[x] = F[x] + ((x > 0) ? C[x - 1] : 0);
+    wB[x] = B[x] + ((x < p - 1) ? C[x] : 0);
+    w[x] = min(p - 1 - x, m);
+  }
+  auto piece_w = [&](int x, int q) -> int64_t {  // split(F_x,k,q) + split(C_{x-1},k,q)
+    const int64_t f0 = F[x] / k, c0 = (x > 0) ? C[x - 1] / k : 0;
+    return (q < k - 1) ? f0 + c0 : (F[x] - (int64_t)(k - 1) * f0) + ((x > 0) ? C[x - 1] - (int64_t)(k - 1) * c0 : 0);
+  };
+  // micro-batch 0's forwards (all pieces; they only depend on each other)
+  if (s == 0) {
+#pragma unroll
+    for (int x = 0; x < P; ++x)
+      if (x < p) FF[x] = ((x > 0) ? FF[x - 1] : 0) + wF[x];
+  } else {
+#pragma unroll
+    for (int x = 0; x < P; ++x) FF[x] = 0;
+    for (int q = 0; q < k; ++q) {
+#pragma unroll
+      for (int x = 0; x < P; ++x) {
+        if (x < p) {
+          const int64_t wq = piece_w(x, q);
+          if (x == 0) FF[0] = FF[0] + wq;
+          else if (q == 0) FF[x] = FF[x - 1] + wq;
+          else FF[x] = max(FF[x - 1], FF[x]) + wq;
+          PV[x][q] = FF[x];
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int x = 0; x < P; ++x) L[x] = FF[x];
+  const int W0 = min(p - 1, m);
+  for (int y = -W0; y < m; ++y) {
+    int64_t prev_old = 0;
+    int64_t prevPV[kMaxK];
+#pragma unroll
+    for (int x = 0; x < P; ++x) {
+      if (x < p) {
+        const int j = y + w[x];
+        const int64_t old = FF[x];
+        const bool sliced = (j >= 1 && j < m && j < s);
+        int64_t savePV[kMaxK];
+        if (sliced)
+          for (int q = 0; q < k; ++q) savePV[q] = PV[x][q];
+        if (j >= 1 && j < m) {
+          const bool use_old = (x > 0) && (w[x - 1] == w[x] + 1);
+          if (sliced) {
+            int64_t run = L[x];
+            for (int q = 0; q < k; ++q) {
+              int64_t in = run;
+              if (x > 0) {
+                const int64_t cr = use_old ? prevPV[q] : PV[x - 1][q];
+                in = max(cr, in);
+              }
+              run = in + piece_w(x, q);
+              PV[x][q] = run;
+            }
+            FF[x] = run;
+            L[x] = run;
+          } else {
+            const int64_t in = L[x];
+            int64_t v;
+            if (x == 0) {
+              v = in + wF[0];
+            } else {
+              const int64_t cr = use_old ? prev_old : FF[x - 1];
+              v = max(cr, in) + wF[x];
+            }
+            FF[x] = v;
+            L[x] = v;
+          }
+        }
+        prev_old = old;
+        if (sliced) {
+          for (int q = 0; q < k; ++q) prevPV[q] = savePV[q];
+        } else {
+          for (int q = 0; q < k; ++q) prevPV[q] = PV[x][q];
+        }
+      }
+    }
+    if (y >= 0) {
+      int64_t bprev = 0;
+#pragma unroll
+      for (int x = P - 1; x >= 0; --x) {
+        if (x < p) {
+          const int64_t in = L[x];
+          const int64_t v = (x == p - 1) ? in + wB[x] : max(bprev, in) + wB[x];
+          L[x] = v;
+          bprev = v;
+        }
+      }
+    }
+  }
+  return L[0];
+}
+
 // Backtrack the unique critical path from B(0, m-1) using the decision bits and
 // return the master stage: most path ops in the 1F1B phase (F(x,j) with j >= w_x,
 // B(x,y) with y < m - w_x; slice pieces count individually), ties -> higher stage,

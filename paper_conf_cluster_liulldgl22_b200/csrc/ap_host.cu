@@ -794,6 +794,76 @@ ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_
   return AP_OK;
 }
 
+ap_status ap_slice_sweep_paper(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                               int32_t k, int32_t s_max, int64_t* time_ns, int32_t* best_s) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (k < 1 || k > AP_MAX_K) return fail(AP_ERR_INVALID, "k=%d", k);
+  if (s_max < 0 || s_max > m) return fail(AP_ERR_INVALID, "s_max=%d outside [0, m]", s_max);
+  if (!time_ns || !best_s || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL argument");
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(internal_stream(plan->device, &s));
+  ap_status res = AP_OK;
+  {
+    Scratch sc(s, plan->pool);
+    int32_t* d_cuts;
+    int64_t* d_T;
+    cudaError_t e = sc.get((void**)&d_cuts, 4 * 32);
+    if (e == cudaSuccess) e = sc.get((void**)&d_T, 8 * (size_t)(s_max + 1));
+    if (e == cudaSuccess && p > 1)
+      e = cudaMemcpyAsync(d_cuts, cuts, 4 * (size_t)(p - 1), cudaMemcpyHostToDevice, s);
+    int launches = 0;
+    if (e == cudaSuccess)
+      e = apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, k, 0,
+                           s_max + 1, d_T, nullptr, s, &launches, 0, 1);
+    if (e == cudaSuccess)
+      e = cudaMemcpyAsync(time_ns, d_T, 8 * (size_t)(s_max + 1), cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "paper slice sweep: %s", cudaGetErrorString(e));
+  }
+  cudaStreamSynchronize(s);
+  if (res != AP_OK) return res;
+  if (time_ns[0] < 0) return fail(AP_ERR_INVALID, "invalid cut vector");
+  int bs = 0;
+  for (int q = 1; q <= s_max; ++q)
+    if (time_ns[q] < time_ns[bs]) bs = q;  // min (T, s)
+  *best_s = bs;
+  return AP_OK;
+}
+
+ap_status ap_slicer_alg2(const ap_plan* plan, int32_t p, const int32_t* cuts, int32_t reading,
+                         int32_t* mb) {
+  g_err.clear();
+  if (!plan) return fail(AP_ERR_INVALID, "plan is NULL");
+  if (p < 1 || p > plan->n || p > AP_MAX_P) return fail(AP_ERR_INVALID, "p=%d", p);
+  if (reading != 0 && reading != 1) return fail(AP_ERR_INVALID, "reading %d", reading);
+  if (!mb || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL argument");
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(internal_stream(plan->device, &s));
+  ap_status res = AP_OK;
+  int32_t h = -1;
+  {
+    Scratch sc(s, plan->pool);
+    int32_t *d_cuts, *d_mb;
+    cudaError_t e = sc.get((void**)&d_cuts, 4 * 32);
+    if (e == cudaSuccess) e = sc.get((void**)&d_mb, 16);
+    if (e == cudaSuccess && p > 1)
+      e = cudaMemcpyAsync(d_cuts, cuts, 4 * (size_t)(p - 1), cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = apk::launch_alg2(plan->dev(), p, d_cuts, reading, d_mb, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&h, d_mb, 4, cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "alg2: %s", cudaGetErrorString(e));
+  }
+  cudaStreamSynchronize(s);
+  if (res != AP_OK) return res;
+  if (h < 0) return fail(AP_ERR_INVALID, "invalid cut vector");
+  *mb = h;
+  return AP_OK;
+}
+
 ap_status ap_critical_path(const ap_plan* plan, int32_t p, int32_t m, int32_t k,
                            const int32_t* cuts, ap_op* ops, int32_t cap, int32_t* len,
                            int32_t* master, int64_t* time_ns) {

@@ -497,6 +497,8 @@ struct EvalArgs {
   int64_t* time_ns;
   int32_t* master;
   uint32_t* gbits;  // global bit scratch when shared memory is too small (or null)
+  int s_const;      // sliced leading micro-batches (1 = micro-batch 0 only, the default)
+  int s_iota;       // 1: row i uses s = i (paper-form slice sweep), k = k_const
 };
 
 template <int P>
@@ -529,13 +531,19 @@ __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
   int c[P + 1];
   const bool okc = load_cuts<P>(A.cuts + (size_t)i * A.cuts_stride, p, n, c);
   const int k = A.kptr ? A.kptr[i] : (A.k_iota ? (int)(i + 1) : A.k_const);
-  if (!okc || k < 1 || k > kMaxK) {
+  const int sl = A.s_iota ? (int)i : A.s_const;
+  if (!okc || k < 1 || k > kMaxK || sl < 0 || sl > A.m) {
     A.time_ns[i] = -1;
     if (A.master) A.master[i] = -1;
     return;
   }
   int64_t F[P], B[P], C[P];
   stage_costs<P>(T, p, c, F, B, C);
+  if (sl != 1) {  // paper Slicer form: T only
+    A.time_ns[i] = sim_sliced<P>(p, m, sl, k, F, B, C);
+    if (A.master) A.master[i] = -1;
+    return;
+  }
   uint32_t pb[P];
   TimesRef not_{nullptr, nullptr, nullptr};
   if (A.master == nullptr) {
@@ -1076,6 +1084,71 @@ __global__ void k_cpath(CpathArgs A) {
   }
 }
 
+// Algorithm 2: the Slicer's analytic number mb of leading
+// micro-batches to slice in halves.  One thread, after the K4 prologue.  Readings
+// (Q22-Q24): x/2 = floor; Comm per boundary (forward hop i->i+1: C_i,
+// gradient hop i->i-1: C_{i-1}); line 21 as printed; endt row p stays 0; stop test
+// reading 0 = pseudocode "tempt <= endt[0][1]", 1 = text "start of the unbroken
+// micro-batch >= end of the second half"; mb stops at p.
+__global__ void k_alg2(DevTables t, int p, const int32_t* cuts, int reading, int32_t* mb_out) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
+  if (threadIdx.x != 0) return;
+  const int n = t.n;
+  int64_t F[kMaxP], Bv[kMaxP], Cv[kMaxP], startt[kMaxP], endt[kMaxP + 1][2];
+  int prev = 0;
+  for (int x = 0; x < p; ++x) {
+    const int hi = (x == p - 1) ? n : cuts[x];
+    if (hi <= prev || hi > n) {
+      *mb_out = -1;
+      return;
+    }
+    F[x] = T.Pf[hi] - T.Pf[prev];
+    Bv[x] = T.Pb[hi] - T.Pb[prev];
+    Cv[x] = (x < p - 1) ? T.comm[hi - 1] : 0;
+    prev = hi;
+  }
+  for (int x = 0; x <= p; ++x) {
+    if (x < p) startt[x] = 0;
+    endt[x][0] = endt[x][1] = 0;
+  }
+  int64_t tempt = 0;
+  int mb = 1;
+  for (int i = 0; i <= p - 2; ++i) tempt += F[i] / 2 + Cv[i] / 2;  // forward fill, halves
+  tempt += F[p - 1] / 2;
+  for (int i = p - 1; i >= 1; --i) {  // backward chain of micro-batch 0
+    tempt += Bv[i] + Cv[i - 1];
+    startt[p - 1 - i] = tempt;
+  }
+  tempt += Bv[0];
+  startt[p - 1] = tempt;
+  for (;;) {
+    for (int i = 0; i <= p - mb; ++i)
+      for (int j = 0; j <= 1; ++j) {
+        int64_t e = endt[i][(j + 1) % 2] + F[i] / 2;
+        if (i > 0) e = max(e, endt[i - 1][j] + F[i - 1] / 2);
+        if (i != p - 1) e += Cv[i] / 2;
+        e = max(e, endt[i + 1][(j + 1) % 2]);
+        endt[i][j] = e;
+      }
+    tempt = startt[mb - 1];
+    for (int i = p - 1 - mb; i >= 1; --i) tempt -= F[i] + Cv[i - 1];
+    tempt -= F[0];
+    const bool stop = (reading == 0) ? (tempt <= endt[0][1]) : (tempt >= endt[0][1]);
+    if (stop || mb >= p) break;
+    ++mb;
+  }
+  *mb_out = mb;
+}
+
+cudaError_t launch_alg2(const DevTables& t, int p, const int32_t* cuts, int reading, int32_t* mb,
+                        cudaStream_t s) {
+  const size_t smem = tables_smem_bytes(t.npad, t.n);
+  k_alg2<<<1, 32, smem, s>>>(t, p, cuts, reading, mb);
+  return cudaGetLastError();
+}
+
 __global__ void k_unrank(DevTables t, int p, uint64_t rank, int32_t* cuts) {
   if (threadIdx.x != 0 || blockIdx.x != 0) return;
   const int n = t.n;
@@ -1155,8 +1228,10 @@ static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
 cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, const int32_t* cuts,
                         int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
-                        int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches) {
-  EvalArgs A{t, p, m, cuts, cuts_stride, kptr, k_const, k_iota, count, time_ns, master, nullptr};
+                        int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches,
+                        int s_const, int s_iota) {
+  EvalArgs A{t, p, m, cuts, cuts_stride, kptr, k_const, k_iota, count, time_ns, master, nullptr,
+             s_const, s_iota};
   uint32_t* gbits = nullptr;
   if (master) {
     const int rows = m + min(p - 1, m);

@@ -24,7 +24,8 @@ cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, 
 cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, const int32_t* cuts,
                         int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
-                        int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches);
+                        int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches,
+                        int s_const = 1, int s_iota = 0);
 
 struct SweepPlan {
   int fast_u32;   // exact u32 saturating sweep
@@ -68,6 +69,10 @@ cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cuda
 // Decode helper: unrank lex rank -> cut vector int32[p-1].
 cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,
                           cudaStream_t s);
+
+// Algorithm 2 on the device: mb (int32) for one cut vector.
+cudaError_t launch_alg2(const DevTables& t, int p, const int32_t* cuts, int reading, int32_t* mb,
+                        cudaStream_t s);
 
 int num_sms(int device);
 

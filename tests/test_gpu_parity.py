@@ -509,3 +509,47 @@ def test_heuristic_adjust_eq1_random(ap, oracle_mod):
         o = M.heuristic(p, m, 0x5EED, 2, 0, 200, adjust_mode=1)
         assert (kv >> 20, kv & 0xFFFFF) == (o["T"], o["restart"]), (n, p, m)
         assert ap.ap_last_sims() == o["sims"]
+
+
+def test_slice_sweep_paper_vs_oracle(ap, oracle_mod):
+    """Paper Slicer form on the GPU (generic sim with s sliced micro-batches) == oracle,
+    incl. m < p-1, k = 2..4, every s in [0, m]."""
+    rng = np.random.default_rng(41)
+    for trial in range(25):
+        kind = ["uniform", "b3f", "small"][trial % 3]
+        n = int(rng.integers(2, 25))
+        f, b, a = synth.random_tables(trial, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p = int(rng.integers(1, min(n, 16) + 1))
+        m = int(rng.integers(1, 2 * p + 4))
+        k = int(rng.integers(2, 5))
+        cuts = synth.random_cuts(trial, n, p, 1)[0]
+        T, bs = ap.ap_slice_sweep_paper(plan, p, m, cuts, k, m)
+        oT, obs = M.slice_sweep_paper(p, m, cuts, k, m)
+        assert list(T) == list(oT) and bs == obs, (n, p, m, k)
+    for cfg in synth.ALL_CONFIGS:
+        wl = synth.config(cfg)
+        f, b, a = wl.arrays()
+        M = oracle_mod.Model.from_workload(wl)
+        plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+        c, _ = M.alg1(wl.p)
+        T, bs = ap.ap_slice_sweep_paper(plan, wl.p, wl.m, c, 2, wl.p)
+        oT, obs = M.slice_sweep_paper(wl.p, wl.m, c, 2, wl.p)
+        assert list(T) == list(oT) and bs == obs
+        for rd in (0, 1):
+            assert ap.ap_slicer_alg2(plan, wl.p, c, rd) == M.alg2(wl.p, c, rd)
+
+
+def test_alg2_random_vs_oracle(ap, oracle_mod):
+    rng = np.random.default_rng(43)
+    for trial in range(30):
+        n = int(rng.integers(2, 40))
+        f, b, a = synth.random_tables(trial, n, ["uniform", "b3f", "small"][trial % 3])
+        M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+        plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+        p = int(rng.integers(1, min(n, 32) + 1))
+        cuts = synth.random_cuts(trial, n, p, 1)[0]
+        for rd in (0, 1):
+            assert ap.ap_slicer_alg2(plan, p, cuts, rd) == M.alg2(p, cuts, rd), (n, p, rd)

@@ -628,3 +628,48 @@ def test_heuristic_eq1_properties(oracle_mod):
             h2 = M.heuristic_restart(p, m, 0x5EED, 2, r, adjust_mode=1)
             assert (h2["T"], list(h2["cuts"]), h2["sims"]) == (h1["T"], list(h1["cuts"]), h1["sims"])
             assert h1["steps"] <= n * p
+
+
+def test_paper_slicer_form_pins(oracle_mod):
+    """Paper Slicer form (first s micro-batches in k pieces): s=0 is unsliced, s=1 is
+    the north-star form (micro-batch 0 in k pieces), T never increases from s=0 to
+    s=1 (P7), and uniform stages with C=0 reproduce P5 at s=1."""
+    for seed in range(60):
+        n = 4 + seed % 10
+        f, b, a = synth.random_tables(seed, n, "b3f")
+        M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+        p = 1 + seed % min(n, 6)
+        m = p + seed % 5
+        cuts = synth.random_cuts(seed, n, p, 1)[0]
+        T, bs = M.slice_sweep_paper(p, m, cuts, 2, m)
+        assert T[0] == M.T(p, m, cuts, k=1)
+        assert T[1] == M.T(p, m, cuts, k=2)
+        assert T[1] <= T[0]
+        assert T[bs] == min(T) and all(T[s] > T[bs] for s in range(bs))
+
+
+def test_alg2_text_reading_matches_simulation(oracle_mod):
+    """Algorithm 2 is unpinned by the paper, but its purpose is to
+    pick the number of halved micro-batches.  Its text reading (reading 1)
+    attains the simulated minimum of T(s) on all five configs and on >= 95% of random
+    Alg.-1 partitions with m = 2p (the paper's Fig. 10 setting); the printed pseudocode
+    test (reading 0) does not (Q23)."""
+    for cfg in synth.ALL_CONFIGS:
+        wl = synth.config(cfg)
+        M = oracle_mod.Model.from_workload(wl)
+        c, _ = M.alg1(wl.p)
+        T, bs = M.slice_sweep_paper(wl.p, wl.m, c, 2, wl.p)
+        mb = M.alg2(wl.p, c, 1)
+        assert 1 <= mb <= wl.p and T[mb] == T[bs]
+    hit = {0: 0, 1: 0}
+    for seed in range(200):
+        rng = np.random.default_rng(seed)
+        n = int(rng.integers(8, 40))
+        f, b, a = synth.random_tables(seed, n, "b3f")
+        M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+        p = int(np.random.default_rng(seed + 1).integers(2, min(n, 10) + 1))
+        c, _ = M.alg1(p)
+        T, bs = M.slice_sweep_paper(p, 2 * p, c, 2, p)
+        for rd in (0, 1):
+            hit[rd] += int(T[M.alg2(p, c, rd)] == T[bs])
+    assert hit[1] >= 190 and hit[0] < hit[1]

@@ -44,11 +44,11 @@ AP_DEV_INLINE uint32_t divk(uint32_t v, uint32_t k, uint32_t M) {
 AP_DEV_INLINE uint64_t divk(uint64_t v, uint32_t k, uint32_t) { return v / k; }
 
 
-// Integer ops of the sweep.  Written as plain operators: ptxas then fuses the add
-// of the backward chain into the max (VIADDMNMX, ALU pipe) and puts most other adds
-// on IMAD.IADD (FMA pipe).  Forcing every add onto IMAD (mad.lo with an opaque
-// multiplier) or a signed offset form that removes the adds were both measured
-// slower on C4 (profiles/r01_sweep_variants.md).
+// Integer ops of the sweep, as plain operators: ptxas fuses the add of the backward
+// chain into the max (VIADDMNMX, ALU pipe) and puts most other adds on IMAD.IADD (FMA
+// pipe).  The steady step forces its remaining adds onto IMAD (fma_add below); doing
+// that everywhere, or a signed offset form without adds, measured slower on C4
+// (profiles/r01_sweep_variants.md).
 template <typename V>
 struct XOps {
   static AP_DEV_INLINE V mx(V a, V b) { return a > b ? a : b; }
@@ -66,6 +66,24 @@ struct XOps {
 // FF_r[x]) is one fused add+max (VIADDMNMX, ALU pipe).  A step is P-1 ALU
 // instructions plus P IMAD adds (FMA pipe): 2P-1 instructions for the 2P max-plus
 // ops of a row.  State between steps: FF[0..P-1] only.
+// a + b issued on the FMA pipe (IMAD with a multiplier the compiler cannot fold).
+// AP_MSTEP_IMAD = 2 puts every add of the fused steady step there, so a step is P-1
+// VIADDMNMX (ALU) + P IMAD (FMA): C4 258.5 -> 252.1 ms (profiles/r01_sweep_variants.md);
+// 1 = only FF'[0], 0 = let ptxas choose (it moves some adds to ALU IADD3).
+#ifndef AP_MSTEP_IMAD
+#define AP_MSTEP_IMAD 2
+#endif
+template <typename V>
+AP_DEV_INLINE V fma_add(V a, V b, uint32_t one) {
+  if constexpr (sizeof(V) == 4) {
+    uint32_t d;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(d) : "r"(a), "r"(one), "r"(b));
+    return d;
+  } else {
+    return a + b;
+  }
+}
+
 template <int P, typename V>
 AP_DEV_INLINE void mstep(V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V wBF0, uint32_t one) {
   using O = XOps<V>;
@@ -74,13 +92,13 @@ AP_DEV_INLINE void mstep(V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V wBF0,
   } else {
     V nF[P];
     V M = O::amx(FF[P - 1], wB[P - 1], FF[P - 2]);
-    nF[P - 1] = O::ad(M, wF[P - 1], one);
+    nF[P - 1] = (AP_MSTEP_IMAD >= 2) ? fma_add(M, wF[P - 1], one) : O::ad(M, wF[P - 1], one);
 #pragma unroll
     for (int x = P - 3; x >= 0; --x) {
       M = O::amx(M, wB[x + 1], FF[x]);
-      nF[x + 1] = O::ad(M, wF[x + 1], one);
+      nF[x + 1] = (AP_MSTEP_IMAD >= 2) ? fma_add(M, wF[x + 1], one) : O::ad(M, wF[x + 1], one);
     }
-    nF[0] = O::ad(M, wBF0, one);
+    nF[0] = (AP_MSTEP_IMAD >= 1) ? fma_add(M, wBF0, one) : O::ad(M, wBF0, one);
 #pragma unroll
     for (int x = 0; x < P; ++x) FF[x] = nF[x];
   }

@@ -163,6 +163,33 @@ ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, i
                                     int32_t mode, int64_t* key, ap_stream_t stream);
 
 /*
+ * ap_search_exhaustive2 -- the same search as ap_search_exhaustive_mode, reduced as
+ * a two-word key for the cases where T << rb | index does not fit in 63 bits (SURVEY
+ * §8d key packing, NEXT N3 "two-phase key reduction").  Same shard, modes, T_ref
+ * bound and exactness; no RANGE failure from key packing.
+ *   out   device int64[2] (written): out[0] = least T over this shard's candidates
+ *         with T <= T_ref, out[1] = the least index = rank*K + (k - k_lo) among them;
+ *         both INT64_MAX when the shard holds none (it cannot hold the winner).
+ * Each CTA stores its lexicographic min (T, index); one more single-CTA kernel
+ * reduces those records.  Multi-GPU: all_reduce(MIN) a copy of out[0] -> T*, then
+ * ap_key2_select(out, T*, idx) and all_reduce(MIN) idx; decode with ap_decode mode 2.
+ * Synchronises `stream` once (to read T_ref), then launches asynchronously.
+ * Errors as ap_search_exhaustive_mode, minus the key-packing RANGE.
+ */
+ap_status ap_search_exhaustive2(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int32_t mode,
+                                int64_t* out, ap_stream_t stream);
+
+/*
+ * ap_key2_select -- phase 2 of the two-phase reduction, stream-ordered on `stream`:
+ * *idx = local[1] if local[0] == *t_star (and is not INT64_MAX), else INT64_MAX.
+ *   local  device int64[2] from ap_search_exhaustive2; t_star, idx device int64[1].
+ * Errors: INVALID (NULL pointer), CUDA.
+ */
+ap_status ap_key2_select(const int64_t* local, const int64_t* t_star, int64_t* idx,
+                         ap_stream_t stream);
+
+/*
  * ap_search_heuristic -- AutoPipe's boundary-shifting heuristic (PAPER.md:147-198,
  * steps 1, 3, 4; adjust_mode 1 adds step 2 / Eq. (1)), run as
  * independent deterministic restarts r in [r_lo, r_hi), one GPU lane each.
@@ -203,6 +230,9 @@ typedef struct {
  *           re-simulate (T must equal the key's T; master from the critical path).
  *   mode 1: key from ap_search_heuristic(seed, radius, adjust_mode): replay the
  *           winning restart on the device to recover its cut vector.
+ *   mode 2: key = the reduced index rank*K + (k - k_lo) of ap_search_exhaustive2
+ *           (k_lo, k_hi as in the search): unrank and re-simulate; time_ns is the
+ *           re-simulated T (the caller holds T* from phase 1 to compare).
  * INVALID if key == INT64_MAX (empty search) or is not decodable.
  */
 ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int32_t k_lo,
@@ -267,6 +297,22 @@ ap_status ap_critical_path(const ap_plan* plan, int32_t p, int32_t m, int32_t k,
  * the max stage load of that partition.
  */
 ap_status ap_alg1(const ap_plan* plan, int32_t p, int32_t* cuts, int64_t* value);
+
+/*
+ * ap_min_lower_bound -- certified lower bound on the optimum T over every partition
+ * and every slicing k <= K (reading R-LB).
+ * The O11 bound LB_x = fill_x + m(F_x+B_x+C_in+C_out) + sum_{i<x}(B_i+C_i) (PAPER.md:
+ * 113-125: stage x runs m FPs and m BPs with their receives, after its fill and before
+ * the BP chain back to stage 0) is relaxed to depend only on (x, c_x, c_{x+1}), and
+ * min over partitions of max_x of it is a bottleneck DP over (x, c_x, c_{x+1}),
+ * O(p n^2) on one CTA.  Exact min_c max_x LB_x(c) when K = 1 and Comm is uniform.
+ * Blocking.  lb: host int64 (T* >= *lb for every partition, every k <= K);
+ * cuts: host int32[p-1] or NULL, a partition attaining the relaxed bound (smallest
+ * split point on ties).  Errors: INVALID for p outside [1, min(n, AP_MAX_P)], m < 1,
+ * K outside [1, AP_MAX_K].
+ */
+ap_status ap_min_lower_bound(const ap_plan* plan, int32_t p, int32_t m, int32_t K, int64_t* lb,
+                             int32_t* cuts);
 
 /* Details of the last ap_search_exhaustive launch on this thread (for benches):
  * which sweep variant ran and its grid. */

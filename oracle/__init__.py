@@ -63,6 +63,8 @@ def _load():
             lib.or_alg1_table.argtypes = [i32, P(i64), P(i64), i32, P(i64), P(i32)]
             lib.or_alg1_reconstruct.restype = i32
             lib.or_alg1_reconstruct.argtypes = [P(i32), i32, i32, i32, i32, P(i32)]
+            lib.or_min_lb.restype = i32
+            lib.or_min_lb.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, i32, P(i64), P(i32)]
             lib.or_count.restype = u64
             lib.or_count.argtypes = [i32, i32]
             lib.or_rank.restype = u64
@@ -221,6 +223,16 @@ class Model:
         c = _i32(cuts)
         return lib.or_lower_bound(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
                                   _p(self.comm, C.c_int64), p, m, K, _p(c, C.c_int32))
+
+    def min_lower_bound(self, p, m, K=1):
+        """Certified minLB over all partitions and k <= K (DESIGN.md
+        reading R-LB): returns (lb, cuts of an argmin partition of the relaxed bound)."""
+        lib = _load()
+        lb = C.c_int64()
+        cuts = np.zeros(max(p - 1, 1), np.int32)
+        _chk(lib.or_min_lb(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                           _p(self.comm, C.c_int64), p, m, K, C.byref(lb), _p(cuts, C.c_int32)))
+        return lb.value, cuts[: p - 1].copy()
 
     def exhaustive_bnb(self, p, m, k_lo=1, k_hi=1, incumbent: Optional[int] = None):
         lib = _load()

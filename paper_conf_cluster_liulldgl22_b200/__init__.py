@@ -23,6 +23,7 @@ AP_MAX_P = 32
 AP_MAX_K = 16
 AP_MAX_N = 512
 INT64_MAX = (1 << 63) - 1
+AP_OK, AP_ERR_INVALID, AP_ERR_RANGE, AP_ERR_CUDA, AP_ERR_NOMEM, AP_ERR_CAPACITY = range(6)
 
 _STATUS = {0: "AP_OK", 1: "AP_ERR_INVALID", 2: "AP_ERR_RANGE", 3: "AP_ERR_CUDA",
            4: "AP_ERR_NOMEM", 5: "AP_ERR_CAPACITY"}
@@ -89,6 +90,12 @@ def _load_lib():
                                      P(i64)]
     lib.ap_alg1.restype = i32
     lib.ap_alg1.argtypes = [vp, i32, P(i32), P(i64)]
+    lib.ap_search_exhaustive2.restype = i32
+    lib.ap_search_exhaustive2.argtypes = [vp, i32, i32, i32, i32, u64, u64, i32, vp, vp]
+    lib.ap_key2_select.restype = i32
+    lib.ap_key2_select.argtypes = [vp, vp, vp, vp]
+    lib.ap_min_lower_bound.restype = i32
+    lib.ap_min_lower_bound.argtypes = [vp, i32, i32, i32, P(i64), P(i32)]
     lib.ap_last_launch.restype = None
     lib.ap_last_launch.argtypes = [P(ApLaunchInfo)]
     lib.ap_last_kernel_ms.restype = i32
@@ -103,9 +110,10 @@ lib = _load_lib()
 # every symbol include/ap.h declares (checked by tests/test_abi.py)
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
            "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_exhaustive_mode",
+           "ap_search_exhaustive2", "ap_key2_select",
            "ap_search_heuristic",
            "ap_decode", "ap_slice_sweep", "ap_slice_sweep_paper", "ap_slicer_alg2",
-           "ap_critical_path", "ap_alg1", "ap_last_launch",
+           "ap_critical_path", "ap_alg1", "ap_min_lower_bound", "ap_last_launch",
            "ap_last_kernel_ms", "ap_last_sims")
 
 
@@ -122,7 +130,7 @@ def _i32(a) -> np.ndarray:
     return np.ascontiguousarray(np.asarray(a, dtype=np.int32))
 
 
-def _ptr(t, dtype_name: str, device_index: Optional[int] = None):
+def _ptr(t, dtype_name: str, device_index: Optional[int] = None, min_numel: int = 0):
     """data_ptr of a contiguous CUDA torch tensor of the given dtype (or None)."""
     if t is None:
         return None
@@ -134,6 +142,8 @@ def _ptr(t, dtype_name: str, device_index: Optional[int] = None):
         raise TypeError(f"expected a contiguous {dtype_name} tensor, got {t.dtype}")
     if device_index is not None and t.device.index != device_index:
         raise ValueError(f"tensor on cuda:{t.device.index}, plan on cuda:{device_index}")
+    if t.numel() < min_numel:
+        raise ValueError(f"expected at least {min_numel} elements, got {t.numel()}")
     return C.c_void_p(t.data_ptr())
 
 
@@ -233,6 +243,21 @@ def ap_search_exhaustive_mode(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, 
                                          _ptr(key, "int64", plan.device), _stream(stream)))
 
 
+def ap_search_exhaustive2(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank_lo: int,
+                          rank_hi: int, mode: int, out, stream=None):
+    """Two-word reduction: out (device int64[2]) = (least T, least index with it)."""
+    _check(lib.ap_search_exhaustive2(plan.handle, int(p), int(m), int(k_lo), int(k_hi),
+                                     int(rank_lo), int(rank_hi), int(mode),
+                                     _ptr(out, "int64", plan.device, 2), _stream(stream)))
+
+
+def ap_key2_select(local, t_star, idx, stream=None):
+    """idx = local[1] if local[0] == t_star else INT64_MAX (device, stream-ordered)."""
+    dev = local.device.index
+    _check(lib.ap_key2_select(_ptr(local, "int64", dev, 2), _ptr(t_star, "int64", dev),
+                              _ptr(idx, "int64", dev), _stream(stream)))
+
+
 def ap_search_heuristic(plan: Plan, p: int, m: int, seed: int, radius: int, r_lo: int,
                         r_hi: int, adjust_mode: int, key, stream=None):
     _check(lib.ap_search_heuristic(plan.handle, int(p), int(m), int(seed), int(radius),
@@ -302,6 +327,16 @@ def ap_alg1(plan: Plan, p: int):
     _check(lib.ap_alg1(plan.handle, int(p), cuts.ctypes.data_as(C.POINTER(C.c_int32)),
                        C.byref(v)))
     return cuts[: p - 1].copy(), v.value
+
+
+def ap_min_lower_bound(plan: Plan, p: int, m: int, K: int = 1):
+    """Certified lower bound on T* over all partitions and k <= K (include/ap.h).
+    Returns (lb, cuts of a partition attaining the relaxed bound)."""
+    cuts = np.zeros(AP_MAX_P, np.int32)
+    v = C.c_int64()
+    _check(lib.ap_min_lower_bound(plan.handle, int(p), int(m), int(K), C.byref(v),
+                                  cuts.ctypes.data_as(C.POINTER(C.c_int32))))
+    return v.value, cuts[: p - 1].copy()
 
 
 def ap_last_launch() -> dict:

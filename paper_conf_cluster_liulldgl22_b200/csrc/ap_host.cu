@@ -449,13 +449,56 @@ ap_status ap_alg1(const ap_plan* plan, int32_t p, int32_t* cuts, int64_t* value)
     if (st == AP_OK) {
       int64_t v = 0;
       std::vector<int32_t> hc(32, 0);
-      cudaError_t e = cudaMemcpyAsync(hc.data(), dc, 4 * 32, cudaMemcpyDeviceToHost, s);
+      cudaError_t e = cudaSuccess;
+      if (p > 1) e = cudaMemcpyAsync(hc.data(), dc, 4 * (size_t)(p - 1), cudaMemcpyDeviceToHost, s);
       if (e == cudaSuccess) e = cudaMemcpyAsync(&v, dv, 8, cudaMemcpyDeviceToHost, s);
       if (e == cudaSuccess) e = cudaStreamSynchronize(s);
       if (e != cudaSuccess) st = fail(AP_ERR_CUDA, "alg1: %s", cudaGetErrorString(e));
       else {
         if (cuts && p > 1) memcpy(cuts, hc.data(), 4 * (p - 1));
         if (value) *value = v;
+      }
+    }
+  }
+  cudaStreamSynchronize(s);
+  return st;
+}
+
+ap_status ap_min_lower_bound(const ap_plan* plan, int32_t p, int32_t m, int32_t K, int64_t* lb,
+                             int32_t* cuts) {
+  g_err.clear();
+  // every stage term is <= LB_x(c) <= T(c) for a partition c holding that stage,
+  // so the plan's overflow guard covers the DP
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (K < 1 || K > AP_MAX_K) return fail(AP_ERR_INVALID, "K=%d outside [1, %d]", K, AP_MAX_K);
+  if (!lb) return fail(AP_ERR_INVALID, "lb is NULL");
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(internal_stream(plan->device, &s));
+  {
+    Scratch sc(s, plan->pool);
+    int16_t* d_arg = nullptr;
+    int32_t* d_cuts = nullptr;
+    int64_t* d_v = nullptr;
+    cudaError_t e = sc.get((void**)&d_arg, (size_t)(plan->n + 1) * (p + 1) * 2);
+    if (e == cudaSuccess) e = sc.get((void**)&d_cuts, 4 * 32);
+    if (e == cudaSuccess) e = sc.get((void**)&d_v, 8);
+    if (e != cudaSuccess) {
+      st = fail(AP_ERR_NOMEM, "minlb scratch");
+    } else {
+      int32_t hc[32] = {0};
+      int64_t v = 0;
+      e = apk::launch_minlb(plan->dev(), p, m, K, d_arg, d_cuts, d_v, s);
+      if (e == cudaSuccess && p > 1)
+        e = cudaMemcpyAsync(hc, d_cuts, 4 * (size_t)(p - 1), cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&v, d_v, 8, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess) {
+        st = fail(AP_ERR_CUDA, "minlb: %s", cudaGetErrorString(e));
+      } else {
+        *lb = v;
+        if (cuts && p > 1) memcpy(cuts, hc, 4 * (size_t)(p - 1));
       }
     }
   }
@@ -470,15 +513,20 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
                                    stream);
 }
 
-ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
-                                    int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
-                                    int32_t mode, int64_t* key, ap_stream_t stream) {
+}  // extern "C"
+
+namespace {
+
+// Shared by the packed-key and the two-phase entry points: exactly one of key / out2.
+ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                 int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int32_t mode,
+                                 int64_t* key, int64_t* out2, ap_stream_t stream) {
   g_err.clear();
   if (mode < AP_SEARCH_FULL || mode > AP_SEARCH_PRUNED)
     return fail(AP_ERR_INVALID, "search mode %d", mode);
   ap_status st = check_pm(plan, p, m);
   if (st != AP_OK) return st;
-  if (!key) return fail(AP_ERR_INVALID, "key is NULL");
+  if (!key && !out2) return fail(AP_ERR_INVALID, "key is NULL");
   if (k_lo < 1 || k_hi < k_lo || k_hi > AP_MAX_K)
     return fail(AP_ERR_INVALID, "k range [%d, %d] outside [1, %d]", k_lo, k_hi, AP_MAX_K);
   uint64_t N;
@@ -507,7 +555,7 @@ ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, i
   AP_CUDA(cudaMemcpyAsync(&tref, d_tref, 8, cudaMemcpyDeviceToHost, s));
   AP_CUDA(cudaStreamSynchronize(s));
   if (tref < 0) return fail(AP_ERR_CUDA, "T_ref evaluation failed");
-  if (rb >= 63 || (uint64_t)tref >= ((1ull << (63 - rb)) - 1))
+  if (key && (rb >= 63 || (uint64_t)tref >= ((1ull << (63 - rb)) - 1)))
     return fail(AP_ERR_RANGE, "key packing: T_ref=%lld needs %d bits + %d rank bits > 63",
                 (long long)tref, bitlen((unsigned __int128)tref), rb);
   // exact u32 saturating fast path: S = T_ref + 1.  Between two
@@ -532,11 +580,20 @@ ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, i
   if (ov && strcmp(ov, "int64") == 0) want_u32 = 0;
   if (ov && strcmp(ov, "generic") == 0) { want_u32 = 0; force_generic = 1; }
   apk::SweepPlan sp{};
-  AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), nullptr, s));
+  unsigned long long* rec = nullptr;
+  if (key) {
+    AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), nullptr, s));
+  } else {
+    AP_CUDA(sc.get((void**)&rec, 16 * (size_t)apk::sweep_max_blocks(plan->device)));
+  }
   AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, S, rb, want_u32,
                             clamp_rows, force_generic, mode,
-                            reinterpret_cast<unsigned long long*>(key), s, &sp));
+                            reinterpret_cast<unsigned long long*>(key), s, &sp, rec));
+  if (rec) {
+    AP_CUDA(apk::launch_reduce2(rec, sp.blocks, reinterpret_cast<long long*>(out2), s));
+    ++launches;
+  }
   AP_CUDA(g_timer.record(1, s, plan->device));
   g_timer.sims_on_device = false;
   g_timer.host_sims = (rank_hi - rank_lo) * (uint64_t)(k_hi - k_lo + 1);
@@ -551,6 +608,42 @@ ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, i
   info.clamp_rows = sp.fast_u32 ? clamp_rows : 0;
   info.launches = launches;
   g_last = info;
+  return AP_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                    int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
+                                    int32_t mode, int64_t* key, ap_stream_t stream) {
+  if (!key) {
+    g_err.clear();
+    return fail(AP_ERR_INVALID, "key is NULL");
+  }
+  return search_exhaustive_impl(plan, p, m, k_lo, k_hi, rank_lo, rank_hi, mode, key, nullptr,
+                                stream);
+}
+
+ap_status ap_search_exhaustive2(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int32_t mode,
+                                int64_t* out, ap_stream_t stream) {
+  if (!out) {
+    g_err.clear();
+    return fail(AP_ERR_INVALID, "out is NULL");
+  }
+  return search_exhaustive_impl(plan, p, m, k_lo, k_hi, rank_lo, rank_hi, mode, nullptr, out,
+                                stream);
+}
+
+ap_status ap_key2_select(const int64_t* local, const int64_t* t_star, int64_t* idx,
+                         ap_stream_t stream) {
+  g_err.clear();
+  if (!local || !t_star || !idx) return fail(AP_ERR_INVALID, "NULL pointer");
+  AP_CUDA(apk::launch_key2_select(reinterpret_cast<const long long*>(local),
+                                  reinterpret_cast<const long long*>(t_star),
+                                  reinterpret_cast<long long*>(idx), S_(stream)));
   return AP_OK;
 }
 
@@ -655,7 +748,8 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
     if (e == cudaSuccess) e = sc.get((void**)&d_master, 16);
     if (e == cudaSuccess) e = sc.get((void**)&d_T, 16);
     if (e != cudaSuccess) res = fail(AP_ERR_NOMEM, "decode scratch");
-    if (res == AP_OK && mode == 0) {
+    bool checkT = true;
+    if (res == AP_OK && (mode == 0 || mode == 2)) {
       uint64_t N;
       res = ap_count(plan->n, p, &N);
       if (res == AP_OK) {
@@ -664,8 +758,14 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
       if (res == AP_OK) {
         const uint64_t K = (uint64_t)(k_hi - k_lo + 1);
         const int rb = bitlen((unsigned __int128)N * K - 1);
-        keyT = (int64_t)((uint64_t)key >> rb);
-        const uint64_t idx = (uint64_t)key & ((rb == 0) ? 0ull : ((1ull << rb) - 1));
+        uint64_t idx;
+        if (mode == 0) {
+          keyT = (int64_t)((uint64_t)key >> rb);
+          idx = (uint64_t)key & ((rb == 0) ? 0ull : ((1ull << rb) - 1));
+        } else {  // two-phase: the key is the index itself (ap_search_exhaustive2)
+          idx = (uint64_t)key;
+          checkT = false;
+        }
         const uint64_t rank = idx / K;
         kk = k_lo + (int)(idx % K);
         if (rank >= N) res = fail(AP_ERR_INVALID, "rank %llu >= N", (unsigned long long)rank);
@@ -726,7 +826,8 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
       int32_t hc[32] = {0};
       int64_t T = -1;
       int32_t M = -1;
-      if (e == cudaSuccess) e = cudaMemcpyAsync(hc, d_cuts, 4 * 32, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess && p > 1)
+        e = cudaMemcpyAsync(hc, d_cuts, 4 * (size_t)(p - 1), cudaMemcpyDeviceToHost, s);
       if (e == cudaSuccess) e = cudaMemcpyAsync(&T, d_T, 8, cudaMemcpyDeviceToHost, s);
       if (e == cudaSuccess) e = cudaMemcpyAsync(&M, d_master, 4, cudaMemcpyDeviceToHost, s);
       if (e == cudaSuccess) e = cudaStreamSynchronize(s);
@@ -736,7 +837,7 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
         if (p > 1) memcpy(out->cuts, hc, 4 * (p - 1));
         out->time_ns = T;
         out->master = M;
-        if (T != keyT)
+        if (checkT && T != keyT)
           res = fail(AP_ERR_INVALID, "key does not decode: T(key)=%lld, re-simulated %lld",
                      (long long)keyT, (long long)T);
         if (mode == 1 && res == AP_OK) {

@@ -256,6 +256,7 @@ struct SweepArgs {
   int clamp_rows;  // u32 path: rows between saturating clamps (>= 1)
   uint32_t one;    // = 1 (adds are plain operators; kept for the XOps interface)
   int mode;        // 0 full, 1 k-factored, 2 k-factored + lower-bound skipping
+  unsigned long long* rec;  // two-phase: per-CTA (T, index) records instead of `key`
 };
 
 AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
@@ -277,6 +278,100 @@ AP_DEV_INLINE void block_min_atomic(unsigned long long v, unsigned long long* ou
     for (int o = 16; o >= 1; o >>= 1) v = min(v, __shfl_xor_sync(0xffffffffu, v, o));
     if (lane == 0 && v != 0x7fffffffffffffffull) atomicMin(out, v);
   }
+}
+
+// Two-phase reduction (NEXT N3): the CTA's lexicographic min of (T, index) stored
+// as record rec[2*blockIdx.x .. +1]; k_reduce2 then reduces the records.
+AP_DEV_INLINE void block_lexmin_store(unsigned long long t, unsigned long long i,
+                                      unsigned long long* rec) {
+  __shared__ unsigned long long s_t[32], s_i[32];
+#pragma unroll
+  for (int o = 16; o >= 1; o >>= 1) {
+    const unsigned long long ot = __shfl_xor_sync(0xffffffffu, t, o);
+    const unsigned long long oi = __shfl_xor_sync(0xffffffffu, i, o);
+    if (ot < t || (ot == t && oi < i)) {
+      t = ot;
+      i = oi;
+    }
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) {
+    s_t[warp] = t;
+    s_i[warp] = i;
+  }
+  __syncthreads();
+  if (warp == 0) {
+    const int nw = (blockDim.x + 31) >> 5;
+    t = (lane < nw) ? s_t[lane] : 0x7fffffffffffffffull;
+    i = (lane < nw) ? s_i[lane] : 0x7fffffffffffffffull;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) {
+      const unsigned long long ot = __shfl_xor_sync(0xffffffffu, t, o);
+      const unsigned long long oi = __shfl_xor_sync(0xffffffffu, i, o);
+      if (ot < t || (ot == t && oi < i)) {
+        t = ot;
+        i = oi;
+      }
+    }
+    if (lane == 0) {
+      rec[2 * (size_t)blockIdx.x] = t;
+      rec[2 * (size_t)blockIdx.x + 1] = i;
+    }
+  }
+}
+
+// Sweep epilogue: one packed key (T << rb | index) or, two-phase, a (T, index) record.
+AP_DEV_INLINE void sweep_result(const SweepArgs& A, bool found, uint64_t T, uint64_t idx) {
+  if (A.rec) {
+    block_lexmin_store(found ? T : 0x7fffffffffffffffull, found ? idx : 0x7fffffffffffffffull,
+                       A.rec);
+  } else {
+    block_min_atomic(found ? ((T << A.rb) | idx) : 0x7fffffffffffffffull, A.key);
+  }
+}
+
+// out[0] = min T over the records, out[1] = least index among the records with that T.
+__global__ void __launch_bounds__(256) k_reduce2(const unsigned long long* rec, int nrec,
+                                                 long long* out) {
+  unsigned long long t = 0x7fffffffffffffffull, i = 0x7fffffffffffffffull;
+  for (int r = threadIdx.x; r < nrec; r += blockDim.x) {
+    const unsigned long long rt = rec[2 * (size_t)r], ri = rec[2 * (size_t)r + 1];
+    if (rt < t || (rt == t && ri < i)) {
+      t = rt;
+      i = ri;
+    }
+  }
+  __shared__ unsigned long long s_t[32], s_i[32];
+#pragma unroll
+  for (int o = 16; o >= 1; o >>= 1) {
+    const unsigned long long ot = __shfl_xor_sync(0xffffffffu, t, o);
+    const unsigned long long oi = __shfl_xor_sync(0xffffffffu, i, o);
+    if (ot < t || (ot == t && oi < i)) {
+      t = ot;
+      i = oi;
+    }
+  }
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (lane == 0) {
+    s_t[warp] = t;
+    s_i[warp] = i;
+  }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    for (int w = 1; w < (int)(blockDim.x >> 5); ++w)
+      if (s_t[w] < t || (s_t[w] == t && s_i[w] < i)) {
+        t = s_t[w];
+        i = s_i[w];
+      }
+    out[0] = (long long)t;
+    out[1] = (long long)i;
+  }
+}
+
+// Phase 2 of the multi-GPU two-phase reduction: this GPU's index if its T is T*.
+__global__ void k_key2_select(const long long* local, const long long* t_star, long long* idx) {
+  *idx = (local[0] == *t_star && local[0] != 0x7fffffffffffffffll) ? local[1]
+                                                                    : 0x7fffffffffffffffll;
 }
 
 template <int P, typename V>
@@ -423,10 +518,7 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
       }
     }
   }
-  const unsigned long long key = (bestT < S)
-                                     ? (((unsigned long long)bestT << A.rb) | bestIdx)
-                                     : 0x7fffffffffffffffull;
-  block_min_atomic(key, A.key);
+  sweep_result(A, bestT < S, (uint64_t)bestT, bestIdx);
 }
 
 // Generic exhaustive sweep: runtime p <= P, any m, exact int64.
@@ -494,10 +586,7 @@ __global__ void __launch_bounds__(128) k_sweep_generic(SweepArgs A) {
       }
     }
   }
-  const unsigned long long key = (bestT < (int64_t)A.S)
-                                     ? (((unsigned long long)bestT << A.rb) | bestIdx)
-                                     : 0x7fffffffffffffffull;
-  block_min_atomic(key, A.key);
+  sweep_result(A, bestT < (int64_t)A.S, (uint64_t)bestT, bestIdx);
 }
 
 __global__ void k_init_key(unsigned long long* key) { *key = 0x7fffffffffffffffull; }
@@ -639,6 +728,86 @@ __global__ void __launch_bounds__(256) k_alg1(DevTables t, int p, int16_t* arg, 
       const int st = arg[e * P1 + jj];
       cuts[jj - 2] = st;
       e = st;
+    }
+  }
+}
+
+// ===========================================================================
+// Certified minLB (reading R-LB), one CTA.  Per-stage
+// relaxation of the O11 bound, g(x, a, b) for stage x = [a, b):
+//   ceil+((Pf[a] - x(K-1)) / K) + (x-1) floor(cmin/K)              (fill)
+//   + m (F + B + [x>0] comm[a-1] + [x<p-1] comm[b-1])              (busy)
+//   + Pb[a] + [x>0] (comm[a-1] + (x-1) cmin)                       (tail)
+// bottleneck DP D[x+1][b] = min_a max(D[x][a], g), a ascending, strict '<'.
+AP_DEV_INLINE int64_t minlb_term(const Tables& T, int p, int m, int K, int64_t cmin, int x,
+                                 int a, int b) {
+  int64_t fill = T.Pf[a] - (int64_t)x * (K - 1);
+  fill = fill <= 0 ? 0 : (fill + K - 1) / K;
+  const int64_t cin = x > 0 ? T.comm[a - 1] : 0;
+  const int64_t cout = x < p - 1 ? T.comm[b - 1] : 0;
+  if (x > 0) fill += (int64_t)(x - 1) * (cmin / K);
+  const int64_t busy = (int64_t)m * (T.Pf[b] - T.Pf[a] + T.Pb[b] - T.Pb[a] + cin + cout);
+  const int64_t tail = T.Pb[a] + (x > 0 ? cin + (int64_t)(x - 1) * cmin : 0);
+  return fill + busy + tail;
+}
+
+__global__ void __launch_bounds__(256) k_minlb(DevTables t, int p, int m, int K, int16_t* arg,
+                                               int32_t* cuts, int64_t* value) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
+  const int n = t.n, N1 = n + 1;
+  int64_t* D = reinterpret_cast<int64_t*>(smem + ((used + 15) & ~size_t(15)));
+  __shared__ int64_t s_cmin;
+  for (int e = threadIdx.x; e < (p + 1) * N1; e += blockDim.x) {
+    D[e] = (e == 0) ? 0 : INT64_MAX;
+    arg[e] = -1;
+  }
+  if (threadIdx.x == 0) {
+    int64_t c = 0;
+    for (int i = 0; i + 1 < n; ++i) c = (i == 0 || T.comm[i] < c) ? T.comm[i] : c;
+    s_cmin = c;
+  }
+  __syncthreads();
+  const int64_t cmin = s_cmin;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int x = 0; x < p; ++x) {
+    const int b_lo = (x == p - 1) ? n : x + 1, b_hi = n - (p - 1 - x);
+    for (int b = b_lo + warp; b <= b_hi; b += nw) {
+      int64_t bv = INT64_MAX;
+      int ba = INT32_MAX;
+      for (int a = x + lane; a < b; a += 32) {
+        const int64_t prev = D[x * N1 + a];
+        if (prev == INT64_MAX) continue;
+        const int64_t g = minlb_term(T, p, m, K, cmin, x, a, b);
+        const int64_t v = prev > g ? prev : g;
+        if (v < bv) {  // a ascending within the lane: first wins
+          bv = v;
+          ba = a;
+        }
+      }
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) {
+        const int64_t ov = __shfl_xor_sync(0xffffffffu, bv, o);
+        const int oa = __shfl_xor_sync(0xffffffffu, ba, o);
+        if (ov < bv || (ov == bv && oa < ba)) {
+          bv = ov;
+          ba = oa;
+        }
+      }
+      if (lane == 0 && bv != INT64_MAX) {
+        D[(x + 1) * N1 + b] = bv;
+        arg[(x + 1) * N1 + b] = (int16_t)ba;
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    *value = D[p * N1 + n];
+    int e = n;
+    for (int x = p; x >= 2; --x) {
+      e = arg[x * N1 + e];
+      cuts[x - 2] = e;
     }
   }
 }
@@ -1214,6 +1383,16 @@ cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, 
   return cudaGetLastError();
 }
 
+cudaError_t launch_minlb(const DevTables& t, int p, int m, int K, int16_t* arg, int32_t* cuts,
+                         int64_t* value, cudaStream_t s) {
+  const size_t smem = ((tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15)) +
+                      (size_t)(t.n + 1) * (p + 1) * 8;
+  cudaError_t e = set_smem((const void*)k_minlb, smem);
+  if (e != cudaSuccess) return e;
+  k_minlb<<<1, 256, smem, s>>>(t, p, m, K, arg, cuts, value);
+  return cudaGetLastError();
+}
+
 template <int P>
 static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   EvalArgs A = A0;
@@ -1274,6 +1453,8 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
   return e;
 }
 
+int sweep_max_blocks(int dev);
+
 template <int P, typename V>
 static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int dev) {
   const size_t smem = tables_smem_bytes(A.t.npad, A.t.n) + (size_t)(3 * (A.t.n + 1) + 4) * sizeof(V);
@@ -1291,6 +1472,7 @@ static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int
   if (A.chunk == 0) A.chunk = 1;
   const uint64_t nthreads = (nr + A.chunk - 1) / A.chunk;
   const uint64_t blocks = (nthreads + threads - 1) / threads;
+  if (A.rec && blocks > (uint64_t)sweep_max_blocks(dev)) return cudaErrorInvalidValue;
   k_sweep_exact<P, V><<<(unsigned)blocks, threads, smem, s>>>(A);
   sp->blocks = (int)blocks;
   sp->threads = threads;
@@ -1315,6 +1497,7 @@ static cudaError_t sweep_generic_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, i
   if (A.chunk == 0) A.chunk = 1;
   const uint64_t nthreads = (nr + A.chunk - 1) / A.chunk;
   const uint64_t blocks = (nthreads + threads - 1) / threads;
+  if (A.rec && blocks > (uint64_t)sweep_max_blocks(dev)) return cudaErrorInvalidValue;
   k_sweep_generic<P><<<(unsigned)blocks, threads, smem, s>>>(A);
   sp->blocks = (int)blocks;
   sp->threads = threads;
@@ -1345,6 +1528,20 @@ static cudaError_t sweep_exact_dispatch(int p, int want_u32, const SweepArgs& A,
   }
 }
 
+cudaError_t launch_reduce2(const unsigned long long* rec, int nrec, long long* out,
+                           cudaStream_t s) {
+  k_reduce2<<<1, 256, 0, s>>>(rec, nrec, out);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_key2_select(const long long* local, const long long* t_star, long long* idx,
+                               cudaStream_t s) {
+  k_key2_select<<<1, 1, 0, s>>>(local, t_star, idx);
+  return cudaGetLastError();
+}
+
+int sweep_max_blocks(int dev) { return num_sms(dev) * 32; }
+
 bool has_exact(int p) {
   return (p >= 1 && p <= 8) || p == 10 || p == 12 || p == 16;
 }
@@ -1352,10 +1549,10 @@ bool has_exact(int p) {
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
-                         SweepPlan* sp) {
+                         SweepPlan* sp, unsigned long long* rec) {
   int dev = 0;
   cudaGetDevice(&dev);
-  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u, mode};
+  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u, mode, rec};
   const bool exact = has_exact(p) && m >= p && (!force_generic || mode != 0);
   sp->exact_p = exact ? 1 : 0;
   sp->fast_u32 = (exact && want_u32) ? 1 : 0;

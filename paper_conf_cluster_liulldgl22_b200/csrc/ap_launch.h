@@ -18,6 +18,10 @@ struct DevTables {
 cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, int64_t* value,
                         cudaStream_t s);
 
+// Certified minLB: arg scratch int16[(n+1)*(p+1)], argmin cuts int32[p-1].
+cudaError_t launch_minlb(const DevTables& t, int p, int m, int K, int16_t* arg, int32_t* cuts,
+                         int64_t* value, cudaStream_t s);
+
 // Generic exact evaluation of `count` candidates.  cuts_stride = p-1 (batch) or 0
 // (all rows share one cut vector).  k source: kptr if non-null, else k_iota ? row+1
 // : k_const.  master may be null.  Invalid rows -> time -1, master -1.
@@ -39,7 +43,18 @@ struct SweepPlan {
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
-                         SweepPlan* plan_out);
+                         SweepPlan* plan_out, unsigned long long* rec = nullptr);
+
+// Two-phase reduction (NEXT N3).  With `rec` (u64[2 * sweep_max_blocks(dev)]) passed
+// to launch_sweep, each CTA stores its lexicographic min (T, index) there instead of
+// packing a key; launch_reduce2 reduces plan_out->blocks records into out[0] = T,
+// out[1] = index.  launch_key2_select: *idx = local[1] if local[0] == *t_star else
+// INT64_MAX (the second all-reduce's operand).
+int sweep_max_blocks(int dev);
+cudaError_t launch_reduce2(const unsigned long long* rec, int nrec, long long* out,
+                           cudaStream_t s);
+cudaError_t launch_key2_select(const long long* local, const long long* t_star, long long* idx,
+                               cudaStream_t s);
 
 // Heuristic restarts [r_lo, r_hi); key = min (T << 20 | r).  replay_cuts (int32[p-1])
 // non-null: single-restart replay writing that restart's best cut vector.  counter

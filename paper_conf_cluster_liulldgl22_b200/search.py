@@ -5,7 +5,9 @@ The candidate space is sharded by contiguous lex-rank (or restart) ranges
 int64 key on its GPU; ONE ``all_reduce(MIN)`` of that 8-byte key over NVLink picks
 the global winner, which every rank then decodes independently (no second
 collective).  The reduction is exact because keys order lexicographically by
-(T, rank, k) / (T, restart) -- include/ap.h.
+(T, rank, k) / (T, restart) -- include/ap.h.  When T << rb | index does not fit in
+63 bits, the two-phase form (NEXT N3) reduces T first and then the least index among
+the ranks holding T*: two 8-byte all-reduces instead of one.
 """
 from __future__ import annotations
 
@@ -13,7 +15,8 @@ from typing import Optional
 
 import torch
 
-from . import (INT64_MAX, Plan, ap_count, ap_decode, ap_search_exhaustive,
+from . import (AP_ERR_RANGE, INT64_MAX, APError, Plan, ap_count, ap_decode,
+               ap_key2_select, ap_search_exhaustive, ap_search_exhaustive2,
                ap_search_heuristic)
 
 
@@ -64,24 +67,64 @@ def min_allreduce_key(key: torch.Tensor, dist=None, group=None) -> torch.Tensor:
     return key
 
 
+def two_phase_reduce(local: torch.Tensor, dist=None, group=None, select=None):
+    """Two-phase MIN reduction of per-rank (T, index) pairs (int64[2] tensors):
+    T* = min T; index = min over the ranks whose T == T* (the others contribute
+    INT64_MAX through `select`, default the device kernel ap_key2_select).
+    Returns (T*, index) as Python ints."""
+    select = select or (lambda loc, ts, idx: ap_key2_select(loc, ts, idx))
+    t_star = local[:1].clone()
+    min_allreduce_key(t_star, dist, group)
+    idx = torch.empty(1, dtype=torch.int64, device=local.device)
+    select(local, t_star, idx)
+    min_allreduce_key(idx, dist, group)
+    return int(t_star.item()), int(idx.item())
+
+
 def search_exhaustive(plan: Plan, p: int, m: int, k_lo: int = 1, k_hi: int = 1,
-                      group=None, decode: bool = True, stream=None) -> dict:
+                      group=None, decode: bool = True, stream=None,
+                      two_phase: Optional[bool] = None, mode: int = 0) -> dict:
     """Exact argmin over all C(n-1,p-1) partitions x k in [k_lo,k_hi], sharded over
-    the ranks of the default process group (if initialised)."""
+    the ranks of the default process group (if initialised).  two_phase None: the
+    packed key when it fits, else the two-phase reduction (every rank takes the same
+    branch: T_ref is the same global value on all of them)."""
     rank, world, dist = _world()
     N = ap_count(plan.n, p)
     lo, hi = shard(N, rank, world)
-    key = torch.empty(1, dtype=torch.int64, device=f"cuda:{plan.device}")
+    dev = f"cuda:{plan.device}"
+    out = {"sims": (hi - lo) * (k_hi - k_lo + 1), "total_sims": N * (k_hi - k_lo + 1),
+           "shard": (lo, hi), "two_phase": False}
+    if not two_phase:
+        key = torch.empty(1, dtype=torch.int64, device=dev)
+        try:
+            if hi > lo:
+                from . import ap_search_exhaustive_mode
+                ap_search_exhaustive_mode(plan, p, m, k_lo, k_hi, lo, hi, mode, key, stream=stream)
+            else:
+                key.fill_(INT64_MAX)
+        except APError as e:
+            if two_phase is not None or e.status != AP_ERR_RANGE or "key packing" not in str(e):
+                raise
+            two_phase = True
+    if not two_phase:
+        min_allreduce_key(key, dist, group)
+        kv = int(key.item())
+        out["key"] = kv
+        if decode:
+            out.update(ap_decode(plan, 0, p, m, k_lo, k_hi, key=kv))
+        return out
+    local = torch.empty(2, dtype=torch.int64, device=dev)
     if hi > lo:
-        ap_search_exhaustive(plan, p, m, k_lo, k_hi, lo, hi, key, stream=stream)
+        ap_search_exhaustive2(plan, p, m, k_lo, k_hi, lo, hi, mode, local, stream=stream)
     else:
-        key.fill_(INT64_MAX)
-    min_allreduce_key(key, dist, group)
-    kv = int(key.item())
-    out = {"key": kv, "sims": (hi - lo) * (k_hi - k_lo + 1), "total_sims": N * (k_hi - k_lo + 1),
-           "shard": (lo, hi)}
-    if decode:
-        out.update(ap_decode(plan, 0, p, m, k_lo, k_hi, key=kv))
+        local.fill_(INT64_MAX)
+    T, idx = two_phase_reduce(local, dist, group)
+    out.update({"two_phase": True, "key": idx, "T": T})
+    if decode and idx != INT64_MAX:
+        res = ap_decode(plan, 2, p, m, k_lo, k_hi, key=idx)
+        if res["time_ns"] != T:
+            raise RuntimeError(f"two-phase decode: T*={T}, re-simulated {res['time_ns']}")
+        out.update(res)
     return out
 
 

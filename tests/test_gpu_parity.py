@@ -553,3 +553,138 @@ def test_alg2_random_vs_oracle(ap, oracle_mod):
         cuts = synth.random_cuts(trial, n, p, 1)[0]
         for rd in (0, 1):
             assert ap.ap_slicer_alg2(plan, p, cuts, rd) == M.alg2(p, cuts, rd), (n, p, rd)
+
+
+# --------------------------------------------------------------------------- N3 minLB
+def test_min_lower_bound_vs_oracle(ap, oracle_mod):
+    """ap_min_lower_bound: bit-exact value and argmin cuts vs the oracle's DP, over
+    table kinds, p up to 32, K up to 16, n up to 512 (the AP_MAX_N edge)."""
+    rng = np.random.default_rng(14)
+    cases = [(int(rng.integers(1, 60)), kind) for kind in
+             ["uniform", "b3f", "small", "equal", "huge", "zero"] for _ in range(6)]
+    cases += [(512, "uniform"), (512, "b3f"), (1, "uniform"), (2, "small")]
+    for i, (n, kind) in enumerate(cases):
+        f, b, a = synth.random_tables(1000 + i, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        for p in sorted({1, min(n, 2), int(rng.integers(1, min(n, 32) + 1)), min(n, 32)}):
+            m = int(rng.choice([1, 2, p, 4 * p + 1, 64]))
+            K = int(rng.integers(1, 17))
+            lb, cuts = ap.ap_min_lower_bound(plan, p, m, K)
+            olb, ocuts = M.min_lower_bound(p, m, K)
+            assert lb == olb, (n, kind, p, m, K)
+            assert list(cuts) == list(ocuts), (n, kind, p, m, K)
+
+
+@pytest.mark.parametrize("cfg", [1, 2, 3, 4, 5])
+def test_min_lower_bound_configs(ap, oracle_mod, cfg):
+    """Configs: GPU == oracle, and the bound never exceeds a GPU-found plan's T."""
+    wl = synth.config(cfg)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model.from_workload(wl)
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    K = wl.k_hi if cfg != 5 else 1
+    lb, cuts = ap.ap_min_lower_bound(plan, wl.p, wl.m, K)
+    assert (lb, list(cuts)) == (lambda r: (r[0], list(r[1])))(M.min_lower_bound(wl.p, wl.m, K))
+    c1, _ = ap.ap_alg1(plan, wl.p)
+    assert lb <= M.T(wl.p, wl.m, c1, k=1)
+
+
+def test_min_lower_bound_errors(ap):
+    f, b, a = synth.random_tables(3, 10, "uniform")
+    plan = _plan(ap, f, b, a, synth.link_for("uniform"))
+    for args in [(0, 4, 1), (11, 4, 1), (3, 0, 1), (3, 4, 0), (3, 4, 17)]:
+        with pytest.raises(ap.APError):
+            ap.ap_min_lower_bound(plan, *args)
+
+
+# --------------------------------------------------------------------------- N3 two-phase
+def _search2(ap, plan, p, m, k_lo, k_hi, mode=0, lo=None, hi=None):
+    import torch
+    N = ap.ap_count(plan.n, p)
+    out = torch.empty(2, dtype=torch.int64, device="cuda")
+    ap.ap_search_exhaustive2(plan, p, m, k_lo, k_hi, 0 if lo is None else lo,
+                             N if hi is None else hi, mode, out)
+    torch.cuda.synchronize()
+    return int(out[0].item()), int(out[1].item())
+
+
+@pytest.mark.parametrize("sweep", ["", "int64", "generic"])
+def test_two_phase_vs_oracle_random(ap, oracle_mod, sweep, monkeypatch):
+    """ap_search_exhaustive2 + ap_decode mode 2 == oracle argmin (T, rank, k), every
+    search mode, and == the packed key wherever that fits."""
+    if sweep:
+        monkeypatch.setenv("AP_SWEEP", sweep)
+    rng = np.random.default_rng(23)
+    for trial in range(12):
+        kind = ["uniform", "b3f", "small", "equal"][trial % 4]
+        n = int(rng.integers(3, 18))
+        f, b, a = synth.random_tables(300 + trial, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p = int(rng.integers(1, min(n, 8) + 1))
+        m = int(rng.choice([1, 2, p, p + 3, 12]))
+        k_lo = int(rng.integers(1, 3)); k_hi = k_lo + int(rng.integers(0, 4))
+        K = k_hi - k_lo + 1
+        o = M.exhaustive(p, m, k_lo, k_hi)
+        packed = _search(ap, plan, p, m, k_lo, k_hi)
+        for mode in (0, 1, 2):
+            T, idx = _search2(ap, plan, p, m, k_lo, k_hi, mode)
+            assert (T, idx // K, k_lo + idx % K) == (o["T"], o["rank"], o["k"]), (trial, mode)
+            res = ap.ap_decode(plan, 2, p, m, k_lo, k_hi, key=idx)
+            assert res["time_ns"] == T and res["cuts"] == [int(x) for x in o["cuts"]]
+            from paper_conf_cluster_liulldgl22_b200.search import rank_bits
+            assert packed == (T << rank_bits(ap.ap_count(n, p), K)) | idx
+
+
+def test_two_phase_when_packed_key_does_not_fit(ap, oracle_mod):
+    """T ~ 2^51 with rb = 14: the packed key is RANGE; the two-phase search (and the
+    search_exhaustive orchestration that falls back to it) returns the oracle argmin."""
+    import torch
+    from paper_conf_cluster_liulldgl22_b200.search import search_exhaustive, shard
+    for seed in range(3):
+        f, b, a = synth.random_tables(40 + seed, 30, "uniform", fmax=1 << 44)
+        bw = synth.link_for("uniform")
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p, m, k_lo, k_hi = 4, 16, 1, 4
+        key = torch.empty(1, dtype=torch.int64, device="cuda")
+        with pytest.raises(ap.APError) as ei:
+            ap.ap_search_exhaustive(plan, p, m, k_lo, k_hi, 0, ap.ap_count(30, p), key)
+        assert ei.value.status == ap.AP_ERR_RANGE
+        o = M.exhaustive(p, m, k_lo, k_hi)
+        assert o["T"] >= 1 << 48
+        for mode in (0, 1, 2):
+            T, idx = _search2(ap, plan, p, m, k_lo, k_hi, mode)
+            assert (T, idx // 4, 1 + idx % 4) == (o["T"], o["rank"], o["k"])
+        r = search_exhaustive(plan, p, m, k_lo, k_hi)
+        assert r["two_phase"] and (r["time_ns"], r["rank"], r["k"]) == (o["T"], o["rank"], o["k"])
+        assert r["cuts"] == [int(x) for x in o["cuts"]]
+        # G shards on one GPU combined with the device phase-2 select
+        N = ap.ap_count(30, p)
+        for G in (2, 5):
+            locs = [torch.tensor(_search2(ap, plan, p, m, k_lo, k_hi, 0, *shard(N, g, G)),
+                                 dtype=torch.int64, device="cuda") for g in range(G)]
+            t_star = torch.tensor([min(int(l[0]) for l in locs)], dtype=torch.int64, device="cuda")
+            idxs = []
+            for l in locs:
+                idx = torch.empty(1, dtype=torch.int64, device="cuda")
+                ap.ap_key2_select(l, t_star, idx)
+                idxs.append(int(idx.item()))
+            assert (int(t_star.item()), min(idxs)) == (o["T"], o["rank"] * 4 + o["k"] - 1)
+
+
+@pytest.mark.parametrize("cfg", [2, 3])
+def test_two_phase_configs_match_packed(ap, cfg):
+    """On the configs (where the packed key fits) both reductions pick the same plan."""
+    wl = synth.config(cfg)
+    f, b, a = wl.arrays()
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    N = ap.ap_count(wl.n, wl.p)
+    K = wl.k_hi - wl.k_lo + 1
+    from paper_conf_cluster_liulldgl22_b200.search import rank_bits
+    key = _search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
+    T, idx = _search2(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
+    assert key == (T << rank_bits(N, K)) | idx

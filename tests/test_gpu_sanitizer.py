@@ -1,0 +1,38 @@
+"""compute-sanitizer over one small run of every kernel family (SURVEY §4 layer 5).
+
+tools/sanitize_run.py drives C1/C2 through every entry point in include/ap.h; each
+tool must report zero errors/hazards.
+"""
+import os
+import shutil
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _sanitizer():
+    for c in (shutil.which("compute-sanitizer"), "/usr/local/cuda/bin/compute-sanitizer"):
+        if c and os.path.exists(c):
+            return c
+    return None
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("tool", ["memcheck", "racecheck", "synccheck", "initcheck"])
+def test_compute_sanitizer_clean(tool):
+    san = _sanitizer()
+    if san is None:
+        pytest.skip("compute-sanitizer not found")
+    r = subprocess.run([san, "--tool", tool, "--error-exitcode", "3", "--print-limit", "10",
+                        sys.executable, os.path.join(ROOT, "tools", "sanitize_run.py")],
+                       capture_output=True, text=True, timeout=900, cwd=ROOT)
+    out = r.stdout + r.stderr
+    assert "sanitize run ok" in out, out[-3000:]
+    assert r.returncode == 0, out[-3000:]
+    if tool == "racecheck":
+        assert "0 hazards displayed (0 errors, 0 warnings)" in out, out[-3000:]
+    else:
+        assert "ERROR SUMMARY: 0 errors" in out, out[-3000:]

@@ -20,6 +20,19 @@ def _free_port():
     return port
 
 
+def _two_phase_cases():
+    import numpy as np
+    import synth
+    cases = {}
+    f, b, a = synth.random_tables(5, 12, "equal")
+    cases["equal"] = (f, b, a, synth.link_for("equal"), 3, 4, 1, 2)
+    f, b, a = synth.random_tables(6, 14, "small")
+    cases["small"] = (f, b, a, synth.link_for("small"), 4, 5, 1, 3)
+    f, b, a = synth.random_tables(7, 9, "uniform")
+    cases["tiny"] = (f, b, a, synth.link_for("uniform"), 9, 2, 1, 1)  # N = 1: one rank empty
+    return cases
+
+
 def _worker(rank, world, port, q):
     try:
         os.environ["MASTER_ADDR"] = "127.0.0.1"
@@ -48,6 +61,26 @@ def _worker(rank, world, port, q):
         key = torch.tensor([(h["T"] << 20) | h["restart"]], dtype=torch.int64)
         min_allreduce_key(key, dist)
         out["heur"] = unpack_heuristic_key(int(key.item()))
+        # two-phase reduction (NEXT N3): per-rank (T, index), T* first, then the least
+        # index among the ranks holding T*.  'equal' tables tie across the shards.
+        from paper_conf_cluster_liulldgl22_b200.search import two_phase_reduce
+
+        def cpu_select(loc, ts, idx):
+            hit = int(loc[0]) == int(ts[0]) and int(loc[0]) != INT64_MAX
+            idx.fill_(int(loc[1]) if hit else INT64_MAX)
+
+        tp = {}
+        for name, (f, b, a, bw, p, m, k_lo, k_hi) in _two_phase_cases().items():
+            M = oracle.Model(f, b, a, bw)
+            N = oracle.count(len(f), p)
+            K = k_hi - k_lo + 1
+            lo, hi = shard(N, rank, world)
+            r = M.exhaustive(p, m, k_lo, k_hi, lo, hi) if hi > lo else {"sims": 0}
+            loc = torch.tensor([r["T"], r["rank"] * K + r["k"] - k_lo] if r["sims"]
+                               else [INT64_MAX, INT64_MAX], dtype=torch.int64)
+            T, idx = two_phase_reduce(loc, dist, None, cpu_select)
+            tp[name] = (T, idx // K, k_lo + idx % K)
+        out["two_phase"] = tp
         q.put((rank, out))
         dist.barrier()
         dist.destroy_process_group()
@@ -77,6 +110,9 @@ def test_two_rank_gloo_shard_reduce_decode(oracle_mod):
     wl = synth.config(2)
     o = oracle_mod.Model.from_workload(wl).heuristic(wl.p, wl.m, wl.seed, wl.radius, 0, 256)
     assert res[0]["heur"] == (o["T"], o["restart"])
+    for name, (f, b, a, bw, p, m, k_lo, k_hi) in _two_phase_cases().items():
+        o = oracle_mod.Model(f, b, a, bw).exhaustive(p, m, k_lo, k_hi)
+        assert res[0]["two_phase"][name] == (o["T"], o["rank"], o["k"]), name
 
 
 def test_shard_covers_exactly():

@@ -673,3 +673,50 @@ def test_alg2_text_reading_matches_simulation(oracle_mod):
         for rd in (0, 1):
             hit[rd] += int(T[M.alg2(p, c, rd)] == T[bs])
     assert hit[1] >= 190 and hit[0] < hit[1]
+
+
+# ----------------------------------------------------------------------------- P14
+def test_P14_minlb_relaxation_exact_for_uniform_comm(oracle_mod):
+    """Certified minLB (reading R-LB): with K = 1 and one Comm value for every
+    cut, the per-stage relaxation is exact, so the DP equals brute force
+    min over all C(n-1,p-1) partitions of the O11 bound (or_lower_bound, pinned by P6),
+    and the partition it returns attains it."""
+    for seed in range(120):
+        kind = ["uniform", "b3f", "small", "equal", "huge"][seed % 5]
+        n = 4 + seed % 9
+        f, b, a = synth.random_tables(seed, n, kind)
+        a = np.full(n, int(a[0]), np.int64)
+        M = oracle_mod.Model(f, b, a, synth.link_for(kind))
+        p = 1 + seed % min(n, 5)
+        m = 1 + seed % 7
+        lb, cuts = M.min_lower_bound(p, m, 1)
+        brute = min(M.lower_bound(p, m, 1, list(c))
+                    for c in itertools.combinations(range(1, n), p - 1))
+        assert lb == brute, (seed, lb, brute)
+        assert M.lower_bound(p, m, 1, list(cuts)) == lb
+        assert all(0 < cuts[i] < n for i in range(p - 1))
+        assert all(cuts[i] < cuts[i + 1] for i in range(p - 2))
+
+
+def test_P14_minlb_is_certified(oracle_mod):
+    """For any Comm and any K: minLB <= min_c LB(c, K) <= min over (c, k <= K) of T
+    (brute force), and the C1 bound is tight (= the P15 optimum 49 664)."""
+    tight = 0
+    for seed in range(120):
+        kind = ["uniform", "b3f", "small", "equal", "huge"][seed % 5]
+        n = 4 + seed % 9
+        f, b, a = synth.random_tables(seed, n, kind)
+        M = oracle_mod.Model(f, b, a, synth.link_for(kind))
+        p = 1 + seed % min(n, 5)
+        m = 1 + seed % 7
+        K = 1 + seed % 4
+        lb, _ = M.min_lower_bound(p, m, K)
+        lbc = min(M.lower_bound(p, m, K, list(c))
+                  for c in itertools.combinations(range(1, n), p - 1))
+        opt = M.exhaustive(p, m, 1, K)["T"]
+        assert lb <= lbc <= opt, (seed, lb, lbc, opt)
+        tight += lb == opt
+    assert tight > 10
+    wl = synth.config(1)
+    M = oracle_mod.Model.from_workload(wl)
+    assert M.min_lower_bound(wl.p, wl.m, 1)[0] == 49664 == M.exhaustive(wl.p, wl.m)["T"]

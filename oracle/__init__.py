@@ -91,6 +91,12 @@ def _load():
             lib.or_heuristic_ex.restype = i32
             lib.or_heuristic_ex.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64, i32, u32,
                                             u32, i32, P(i64), P(u32), P(i32), P(i64), P(u64)]
+            lib.or_reach_restart.restype = i32
+            lib.or_reach_restart.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64, i32, u32,
+                                             i32, P(i64), P(i32), P(u64), P(i32)]
+            lib.or_reach.restype = i32
+            lib.or_reach.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64, i32, u32, u32,
+                                     i32, P(i64), P(u32), P(i32), P(u64), P(u32)]
             lib.or_heuristic_restart_ex.restype = i32
             lib.or_heuristic_restart_ex.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, u64,
                                                     i32, u32, i32, P(i64), P(i32), P(u64), P(i32)]
@@ -283,6 +289,41 @@ class Model:
         if per_restart:
             out["per_restart_T"] = per[: r_hi - r_lo].copy()
         return out
+
+    def reach_restart(self, p, m, seed, radius, r, vmax=4096):
+        """Reachable-set search of one restart (NEXT N1, reading R-N1)."""
+        lib = _load()
+        T = C.c_int64(); sims = C.c_uint64(); tr = C.c_int32()
+        cuts = np.zeros(max(p - 1, 1), np.int32)
+        _chk(lib.or_reach_restart(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                                  _p(self.comm, C.c_int64), p, m, seed, radius, r, vmax,
+                                  C.byref(T), _p(cuts, C.c_int32), C.byref(sims), C.byref(tr)))
+        return {"T": T.value, "cuts": cuts[: p - 1].copy(), "sims": sims.value,
+                "truncated": bool(tr.value)}
+
+    def reach(self, p, m, seed, radius, r_lo, r_hi, vmax=4096):
+        lib = _load()
+        T = C.c_int64(); r = C.c_uint32(); sims = C.c_uint64(); tr = C.c_uint32()
+        cuts = np.zeros(max(p - 1, 1), np.int32)
+        _chk(lib.or_reach(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                          _p(self.comm, C.c_int64), p, m, seed, radius, r_lo, r_hi, vmax,
+                          C.byref(T), C.byref(r), _p(cuts, C.c_int32), C.byref(sims),
+                          C.byref(tr)))
+        return {"T": T.value, "restart": r.value, "cuts": cuts[: p - 1].copy(),
+                "sims": sims.value, "truncated": tr.value}
+
+    def reach_parallel(self, p, m, seed, radius, r_lo, r_hi, vmax=4096, threads=None):
+        threads = threads or os.cpu_count() or 1
+        tot = r_hi - r_lo
+        edges = [r_lo + (tot * i) // threads for i in range(threads + 1)]
+        idx = [i for i in range(threads) if edges[i + 1] > edges[i]]
+        with ThreadPoolExecutor(threads) as ex:
+            res = list(ex.map(lambda i: self.reach(p, m, seed, radius, edges[i], edges[i + 1],
+                                                   vmax), idx))
+        best = dict(min(res, key=lambda d: (d["T"], d["restart"])))
+        best["sims"] = sum(d["sims"] for d in res)
+        best["truncated"] = sum(d["truncated"] for d in res)
+        return best
 
     def heuristic_parallel(self, p, m, seed, radius, r_lo, r_hi, threads=None,
                            per_restart: bool = False, adjust_mode: int = 0):

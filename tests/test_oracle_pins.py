@@ -720,3 +720,82 @@ def test_P14_minlb_is_certified(oracle_mod):
     wl = synth.config(1)
     M = oracle_mod.Model.from_workload(wl)
     assert M.min_lower_bound(wl.p, wl.m, 1)[0] == 49664 == M.exhaustive(wl.p, wl.m)["T"]
+
+
+# ----------------------------------------------------------------------------- N1 reach
+def test_reach_is_the_fixpoint_closure(oracle_mod):
+    """Reachable-set search (reading R-N1) against an order-free definition:
+    with T and master of EVERY partition simulated up front (brute force), the
+    evaluated set must be the least set E with start in E and, for every u in the
+    qualifying set Q (start, plus children c of a Q-node u with master(c) <= master(u))
+    with master(u) > 0, all of u's children in E.  The result is min T over E, and it
+    is never worse than the greedy walk (whose path lies inside Q)."""
+    for seed in range(40):
+        kind = ["uniform", "b3f", "small", "equal"][seed % 4]
+        n = 6 + seed % 7
+        f, b, a = synth.random_tables(seed, n, kind)
+        M = oracle_mod.Model(f, b, a, synth.link_for(kind))
+        p = 2 + seed % min(n - 1, 4)
+        m = p + seed % 5
+        allp = {c: M.simulate(p, m, list(c)) for c in itertools.combinations(range(1, n), p - 1)}
+        _, arg = M.alg1_table(p)
+
+        def kids(c, i):
+            cc = [0] + list(c) + [n]
+            out = []
+            if cc[i + 1] - cc[i] < 2:
+                return out
+            A = cc[:]; A[i] += 1; out.append(A)
+            Ap = A[:]
+            e = Ap[i - 1]
+            for jj in range(i - 1, 1, -1):
+                Ap[jj - 1] = int(arg[e, jj]); e = Ap[jj - 1]
+            if Ap != A:
+                out.append(Ap)
+            if i <= p - 2:
+                Bc = cc[:]; Bc[i + 1] -= 1; out.append(Bc)
+                Bp = Bc[:]
+                e = Bp[i]
+                for jj in range(i, 1, -1):
+                    Bp[jj - 1] = int(arg[e, jj]); e = Bp[jj - 1]
+                if Bp != Bc:
+                    out.append(Bp)
+            return [tuple(x[1:p]) for x in out]
+
+        for r in range(4):
+            start = tuple(int(x) for x in M.restart_start(p, seed, 2, r))
+            Q, E, todo = {start}, {start}, [start]
+            while todo:
+                u = todo.pop()
+                iu = allp[u]["master"]
+                if iu == 0:
+                    continue
+                for c in kids(u, iu):
+                    E.add(c)
+                    if allp[c]["master"] <= iu and c not in Q:
+                        Q.add(c); todo.append(c)
+            o = M.reach_restart(p, m, seed, 2, r)
+            assert not o["truncated"]
+            assert o["sims"] == len(E), (seed, r)
+            assert o["T"] == min(allp[c]["T"] for c in E)
+            assert allp[tuple(int(x) for x in o["cuts"])]["T"] == o["T"]
+            assert o["T"] <= M.heuristic_restart(p, m, seed, 2, r)["T"]
+
+
+def test_reach_truncation_and_bounds(oracle_mod):
+    """vmax caps the evaluated set exactly (sims == vmax when truncated); with a cap
+    the result is still an attained T >= the optimum; restart 0 on C2 reaches the
+    k=1 optimum (P15) like the greedy walk."""
+    wl = synth.config(5)
+    M = oracle_mod.Model.from_workload(wl)
+    full = M.reach_restart(wl.p, wl.m, wl.seed, wl.radius, 0)
+    assert not full["truncated"] and full["sims"] > 8
+    for vmax in (1, 2, 5, full["sims"] - 1):
+        o = M.reach_restart(wl.p, wl.m, wl.seed, wl.radius, 0, vmax=vmax)
+        assert o["truncated"] and o["sims"] == vmax and o["T"] >= full["T"]
+        assert M.T(wl.p, wl.m, o["cuts"]) == o["T"]
+    o = M.reach_restart(wl.p, wl.m, wl.seed, wl.radius, 0, vmax=full["sims"])
+    assert not o["truncated"] and o["T"] == full["T"]
+    wl = synth.config(2)
+    M = oracle_mod.Model.from_workload(wl)
+    assert M.reach_restart(wl.p, wl.m, wl.seed, wl.radius, 0)["T"] == 89891590

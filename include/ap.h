@@ -214,6 +214,28 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
                               int32_t radius, uint32_t r_lo, uint32_t r_hi,
                               int32_t adjust_mode, int64_t* key, ap_stream_t stream);
 
+/*
+ * ap_search_reachable -- the literal reading of PAPER.md:196 "partition schemes with a
+ * master <= i will be processed" (reading R-N1): every
+ * qualifying child is processed, not only the best one.  Per restart r (same start as
+ * ap_search_heuristic: Alg. 1 for r = 0, the seeded perturbation otherwise), a
+ * breadth-first search: a scheme with master i > 0 generates its children a, a', b,
+ * b' (as in ap_search_heuristic); a child not evaluated before is simulated and joins
+ * the evaluated set in that order, and joins the queue if its master is <= i.  The
+ * restart stops when the queue is empty or when vmax schemes have been evaluated
+ * (ap_last_truncated counts those).  Its result is the first-evaluated scheme with
+ * the least T; never worse than ap_search_heuristic's greedy walk, whose path lies
+ * inside the evaluated set.  One 4-lane group per restart on the device.
+ *   key   device int64[1]: min over restarts of (T << 20 | r), INT64_MAX if none.
+ *   0 <= r_lo < r_hi <= 2^20, 0 <= radius <= 2^20, 1 <= vmax <= 2^20; k = 1.
+ * Scratch from the plan's pool: (restart groups in flight) x vmax x (2*P + 8) bytes.
+ * Synchronises `stream` once (overflow guard), then launches asynchronously.
+ * Errors: INVALID, RANGE (overflow guard), NOMEM (scratch), CUDA.
+ */
+ap_status ap_search_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
+                              int32_t radius, uint32_t r_lo, uint32_t r_hi, int32_t vmax,
+                              int64_t* key, ap_stream_t stream);
+
 typedef struct {
   int64_t time_ns;          /* T of the decoded candidate                     */
   uint64_t rank;            /* lex rank (mode 0) / rank of the cut vector (1) */
@@ -238,6 +260,14 @@ typedef struct {
 ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int32_t k_lo,
                     int32_t k_hi, uint64_t seed, int32_t radius, int32_t adjust_mode,
                     int64_t key, ap_result* out);
+
+/*
+ * ap_decode_reachable -- decode a key of ap_search_reachable (same seed, radius, vmax):
+ * replays the winning restart on the device, re-simulates its best scheme with the
+ * critical path (T must equal the key's T).  Blocking.  INVALID for an empty key.
+ */
+ap_status ap_decode_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
+                              int32_t radius, int32_t vmax, int64_t key, ap_result* out);
 
 /*
  * ap_slice_sweep -- the Slicer's choice for one partition (§III-C;
@@ -339,6 +369,10 @@ ap_status ap_last_kernel_ms(float* ms);
  * thread: (rank_hi-rank_lo)*(k_hi-k_lo+1) for the sweep; counted on the device for the
  * heuristic (blocks until that kernel has finished). */
 ap_status ap_last_sims(uint64_t* sims);
+
+/* Restarts of the last ap_search_reachable call on this thread that stopped at vmax
+ * evaluated schemes (blocks until that kernel has finished); 0 after any other search. */
+ap_status ap_last_truncated(uint64_t* truncated);
 
 #ifdef __cplusplus
 }

@@ -94,6 +94,12 @@ def _load_lib():
     lib.ap_search_exhaustive2.argtypes = [vp, i32, i32, i32, i32, u64, u64, i32, vp, vp]
     lib.ap_key2_select.restype = i32
     lib.ap_key2_select.argtypes = [vp, vp, vp, vp]
+    lib.ap_search_reachable.restype = i32
+    lib.ap_search_reachable.argtypes = [vp, i32, i32, u64, i32, u32, u32, i32, vp, vp]
+    lib.ap_decode_reachable.restype = i32
+    lib.ap_decode_reachable.argtypes = [vp, i32, i32, u64, i32, i32, i64, P(ApResult)]
+    lib.ap_last_truncated.restype = i32
+    lib.ap_last_truncated.argtypes = [P(u64)]
     lib.ap_min_lower_bound.restype = i32
     lib.ap_min_lower_bound.argtypes = [vp, i32, i32, i32, P(i64), P(i32)]
     lib.ap_last_launch.restype = None
@@ -111,7 +117,8 @@ lib = _load_lib()
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
            "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_exhaustive_mode",
            "ap_search_exhaustive2", "ap_key2_select",
-           "ap_search_heuristic",
+           "ap_search_heuristic", "ap_search_reachable", "ap_decode_reachable",
+           "ap_last_truncated",
            "ap_decode", "ap_slice_sweep", "ap_slice_sweep_paper", "ap_slicer_alg2",
            "ap_critical_path", "ap_alg1", "ap_min_lower_bound", "ap_last_launch",
            "ap_last_kernel_ms", "ap_last_sims")
@@ -263,6 +270,28 @@ def ap_search_heuristic(plan: Plan, p: int, m: int, seed: int, radius: int, r_lo
     _check(lib.ap_search_heuristic(plan.handle, int(p), int(m), int(seed), int(radius),
                                    int(r_lo), int(r_hi), int(adjust_mode),
                                    _ptr(key, "int64", plan.device), _stream(stream)))
+
+
+def ap_search_reachable(plan: Plan, p: int, m: int, seed: int, radius: int, r_lo: int,
+                        r_hi: int, vmax: int, key, stream=None):
+    """Reachable-set (all-children) restarts; key = min (T << 20 | r) (include/ap.h)."""
+    _check(lib.ap_search_reachable(plan.handle, int(p), int(m), int(seed), int(radius),
+                                   int(r_lo), int(r_hi), int(vmax),
+                                   _ptr(key, "int64", plan.device), _stream(stream)))
+
+
+def ap_decode_reachable(plan: Plan, p: int, m: int, seed: int, radius: int, vmax: int,
+                        key: int) -> dict:
+    out = ApResult()
+    _check(lib.ap_decode_reachable(plan.handle, int(p), int(m), int(seed), int(radius),
+                                   int(vmax), int(key), C.byref(out)))
+    return _result(out)
+
+
+def ap_last_truncated() -> int:
+    v = C.c_uint64()
+    _check(lib.ap_last_truncated(C.byref(v)))
+    return v.value
 
 
 def _result(r: ApResult) -> dict:

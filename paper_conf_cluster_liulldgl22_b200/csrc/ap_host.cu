@@ -40,12 +40,14 @@ struct KernelTimer {
         if (r != cudaSuccess) return r;
       }
     armed = (which == 1);
+    if (which == 0) truncated_valid = false;
     return cudaEventRecord(ev[which], s);
   }
   // simulations of the last search: known on the host (exhaustive) or counted on
   // the device (heuristic, d_sims valid once ev[1] has completed)
   uint64_t host_sims = 0;
   bool sims_on_device = false;
+  bool truncated_valid = false;  // the last search was ap_search_reachable
   unsigned long long* d_sims = nullptr;
   int d_sims_dev = -1;
   cudaError_t sims_buffer(int device, unsigned long long** out) {
@@ -720,6 +722,139 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   ap_launch_info info{};
   info.launches = 3;  // alg1, init, restarts
   g_last = info;
+  return AP_OK;
+}
+
+ap_status ap_search_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
+                              int32_t radius, uint32_t r_lo, uint32_t r_hi, int32_t vmax,
+                              int64_t* key, ap_stream_t stream) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (!key) return fail(AP_ERR_INVALID, "key is NULL");
+  if (r_lo >= r_hi || r_hi > (1u << 20)) return fail(AP_ERR_INVALID, "restart range [%u, %u)", r_lo, r_hi);
+  if (radius < 0 || radius > (1 << 20)) return fail(AP_ERR_INVALID, "radius %d", radius);
+  if (vmax < 1 || vmax > (1 << 20)) return fail(AP_ERR_INVALID, "vmax %d outside [1, 2^20]", vmax);
+  cudaStream_t s = S_(stream);
+  DeviceGuard g(plan->device);
+  Scratch sc(s, plan->pool);
+  int16_t* d_arg;
+  int32_t* d_a1;
+  int64_t* d_val;
+  st = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
+  if (st != AP_OK) return st;
+  unsigned int* d_ctr;
+  AP_CUDA(sc.get((void**)&d_ctr, 16));
+  size_t bytes = 0;
+  AP_CUDA(apk::reach_scratch_bytes(plan->dev(), p, m, r_hi - r_lo, vmax, &bytes));
+  void* d_scr = nullptr;
+  if (sc.get(&d_scr, bytes) != cudaSuccess)
+    return fail(AP_ERR_NOMEM, "reachable-set scratch: %zu bytes", bytes);
+  unsigned long long* d_sims = nullptr;
+  AP_CUDA(g_timer.sims_buffer(plan->device, &d_sims));
+  AP_CUDA(cudaMemsetAsync(d_sims, 0, 16, s));
+  AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), d_ctr, s));
+  AP_CUDA(g_timer.record(0, s, plan->device));
+  AP_CUDA(apk::launch_reach(plan->dev(), p, m, seed, radius, r_lo, r_hi, vmax, d_arg, d_a1, d_ctr,
+                            reinterpret_cast<unsigned long long*>(key), d_sims, nullptr, d_scr,
+                            s));
+  AP_CUDA(g_timer.record(1, s, plan->device));
+  g_timer.sims_on_device = true;
+  g_timer.truncated_valid = true;
+  ap_launch_info info{};
+  info.launches = 3;  // alg1, init, search
+  g_last = info;
+  return AP_OK;
+}
+
+ap_status ap_decode_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
+                              int32_t radius, int32_t vmax, int64_t key, ap_result* out) {
+  g_err.clear();
+  ap_status st = check_pm(plan, p, m);
+  if (st != AP_OK) return st;
+  if (!out) return fail(AP_ERR_INVALID, "out is NULL");
+  if (key == INT64_MAX || key < 0) return fail(AP_ERR_INVALID, "empty key (no candidate found)");
+  if (vmax < 1 || vmax > (1 << 20)) return fail(AP_ERR_INVALID, "vmax %d", vmax);
+  memset(out, 0, sizeof *out);
+  out->p = p;
+  out->k = 1;
+  const int64_t keyT = key >> 20;
+  const uint32_t r = (uint32_t)(key & ((1 << 20) - 1));
+  out->restart = r;
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(internal_stream(plan->device, &s));
+  ap_status res = AP_OK;
+  {
+    Scratch sc(s, plan->pool);
+    int16_t* d_arg;
+    int32_t* d_a1;
+    int64_t* d_val;
+    int32_t* d_cuts = nullptr;
+    int32_t* d_master = nullptr;
+    int64_t* d_T = nullptr;
+    unsigned int* d_ctr = nullptr;
+    unsigned long long* d_key = nullptr;
+    void* d_scr = nullptr;
+    size_t bytes = 0;
+    res = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
+    cudaError_t e = cudaSuccess;
+    if (res == AP_OK) {
+      e = sc.get((void**)&d_cuts, 4 * 32);
+      if (e == cudaSuccess) e = sc.get((void**)&d_master, 16);
+      if (e == cudaSuccess) e = sc.get((void**)&d_T, 16);
+      if (e == cudaSuccess) e = sc.get((void**)&d_ctr, 16);
+      if (e == cudaSuccess) e = sc.get((void**)&d_key, 16);
+      if (e == cudaSuccess) e = apk::reach_scratch_bytes(plan->dev(), p, m, 1, vmax, &bytes);
+      if (e == cudaSuccess) e = sc.get(&d_scr, bytes);
+      if (e != cudaSuccess) res = fail(AP_ERR_NOMEM, "decode scratch");
+    }
+    if (res == AP_OK) {
+      // replay restart r alone: its best cut vector (first-evaluated least T)
+      e = apk::launch_init_key(d_key, d_ctr, s);
+      if (e == cudaSuccess)
+        e = apk::launch_reach(plan->dev(), p, m, seed, radius, r, r + 1, vmax, d_arg, d_a1, d_ctr,
+                              d_key, nullptr, p > 1 ? d_cuts : nullptr, d_scr, s);
+      int launches = 0;
+      if (e == cudaSuccess)
+        e = apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, 1,
+                             0, 1, d_T, d_master, s, &launches);
+      int32_t hc[32] = {0};
+      int64_t T = -1;
+      int32_t M = -1;
+      if (e == cudaSuccess && p > 1)
+        e = cudaMemcpyAsync(hc, d_cuts, 4 * (size_t)(p - 1), cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&T, d_T, 8, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaMemcpyAsync(&M, d_master, 4, cudaMemcpyDeviceToHost, s);
+      if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+      if (e != cudaSuccess) {
+        res = fail(AP_ERR_CUDA, "reachable decode: %s", cudaGetErrorString(e));
+      } else {
+        if (p > 1) memcpy(out->cuts, hc, 4 * (p - 1));
+        out->time_ns = T;
+        out->master = M;
+        if (T != keyT)
+          res = fail(AP_ERR_INVALID, "key does not decode: T(key)=%lld, re-simulated %lld",
+                     (long long)keyT, (long long)T);
+      }
+    }
+  }
+  cudaStreamSynchronize(s);
+  return res;
+}
+
+ap_status ap_last_truncated(uint64_t* truncated) {
+  if (!truncated) return fail(AP_ERR_INVALID, "truncated is NULL");
+  if (!g_timer.armed) return fail(AP_ERR_INVALID, "no search launched on this thread");
+  if (!g_timer.truncated_valid) {
+    *truncated = 0;
+    return AP_OK;
+  }
+  cudaError_t e = cudaEventSynchronize(g_timer.ev[1]);
+  unsigned long long v[2] = {0, 0};
+  if (e == cudaSuccess) e = cudaMemcpy(v, g_timer.d_sims, 16, cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return fail(AP_ERR_CUDA, "truncated read: %s", cudaGetErrorString(e));
+  *truncated = v[1];
   return AP_OK;
 }
 

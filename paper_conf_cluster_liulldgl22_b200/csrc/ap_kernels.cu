@@ -1185,6 +1185,257 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
 }
 
 // ===========================================================================
+// K3r reachable-set search (NEXT N1; reading R-N1): the literal reading of
+// PAPER.md:196, every qualifying child is processed.  One QUAD (4 lanes) per restart,
+// breadth-first: the quad pops the next queued scheme with master i > 0, lane q
+// builds child q (a, a', b, b' -- the order of k_heur's gen_child), drops it if it
+// is invalid or already evaluated (a 32-bit hash scan of the quad's evaluated list,
+// then a full compare), and the new children are simulated together.  They join the
+// evaluated list in child order; those with master <= i join the queue.  The outer
+// loop is warp-uniform, so the simulations of all quads of a warp in one iteration
+// run converged.  At most vmax schemes per restart are evaluated (exactly the
+// oracle's cut-off).  Per-quad lists live in global scratch (L1/L2-resident).
+struct ReachArgs {
+  DevTables t;
+  int p, m;
+  uint64_t seed;
+  int radius;
+  uint32_t r_lo, r_hi;
+  const int16_t* arg;
+  const int32_t* alg1;
+  unsigned int* counter;
+  unsigned long long* key;
+  int vmax;
+  int16_t* g_cuts;            // [quads][vmax][P]
+  uint32_t* g_hash;           // [quads][vmax]
+  uint32_t* g_queue;          // [quads][vmax]: node | master << 24
+  unsigned long long* stats;  // optional: [0] simulations, [1] truncated restarts
+  int32_t* replay;            // optional: best cuts of the (single) restart
+};
+
+AP_DEV_INLINE uint32_t cut_hash(const int (&c)[33], int p) {
+  uint32_t h = 0x811c9dc5u;
+  for (int x = 1; x <= p - 1; ++x) h = (h ^ (uint32_t)c[x]) * 0x01000193u;
+  return h;
+}
+
+template <int P>
+__global__ void __launch_bounds__(128) k_reach(ReachArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int n = A.t.n, p = A.p, m = A.m, P1 = p + 1, vmax = A.vmax;
+  int16_t* s_arg = reinterpret_cast<int16_t*>(smem + ((used + 15) & ~size_t(15)));
+  const int narg = (n + 1) * P1;
+  int32_t* s_a1 = reinterpret_cast<int32_t*>(s_arg + ((narg + 7) & ~7));
+  uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_a1 + 32);
+  for (int e = threadIdx.x; e < narg; e += blockDim.x) s_arg[e] = A.arg[e];
+  for (int e = threadIdx.x; e < p - 1; e += blockDim.x) s_a1[e] = A.alg1[e];
+  __syncthreads();
+  BitsRef br{s_bits + threadIdx.x, (int)blockDim.x};
+  TimesRef not_{nullptr, nullptr, nullptr};
+
+  const int lane = threadIdx.x & 31, q = lane & 3, qb = lane & ~3;
+  const unsigned qmask = 0xFu << qb;
+  const size_t quad = ((size_t)blockIdx.x * blockDim.x + threadIdx.x) >> 2;
+  int16_t* Qc = A.g_cuts + quad * (size_t)vmax * P;
+  uint32_t* Qh = A.g_hash + quad * (size_t)vmax;
+  uint32_t* Qq = A.g_queue + quad * (size_t)vmax;
+
+  int phase = 0;  // 0 need a restart, 1 simulate the start, 2 expand, 3 no work left
+  uint32_t r = 0;
+  int nv = 0, qh = 0, qt = 0;
+  bool trunc = false;
+  int64_t bestT = INT64_MAX;
+  int bestNode = 0;
+  unsigned long long lane_key = 0x7fffffffffffffffull, nsims = 0, ntrunc = 0;
+  for (;;) {
+    if (phase == 0) {
+      unsigned int v = 0;
+      if (q == 0) v = atomicAdd(A.counter, 1u);
+      v = __shfl_sync(qmask, v, qb);
+      r = v + A.r_lo;
+      if (r >= A.r_hi || v >= A.r_hi - A.r_lo) {
+        phase = 3;
+      } else {
+        phase = 1;
+        nv = qh = qt = 0;
+        trunc = false;
+        bestT = INT64_MAX;
+        bestNode = 0;
+      }
+    }
+    if (__all_sync(0xffffffffu, phase == 3)) break;
+
+    // ---- this iteration's candidate of this lane
+    int cand[33];
+    cand[0] = 0;
+#pragma unroll
+    for (int x = 1; x <= 32; ++x) cand[x] = n;
+    bool want = false;
+    int slot = 0, parentM = 0;
+    if (phase == 1) {
+      // restart start: Alg. 1 (r = 0) or the seeded perturbation (reading Q21)
+      int prev = 0;
+      for (int x = 1; x <= p - 1; ++x) {
+        int64_t v = s_a1[x - 1];
+        if (r != 0) {
+          const uint64_t u = splitmix64(A.seed ^ ((uint64_t)r << 32) ^ (uint64_t)x);
+          v += (int64_t)(u % (uint64_t)(2 * A.radius + 1)) - A.radius;
+          v = v < prev + 1 ? prev + 1 : v;
+          v = v > n - (p - x) ? n - (p - x) : v;
+        }
+        cand[x] = (int)v;
+        prev = (int)v;
+      }
+      want = (q == 0);
+      slot = 0;
+    } else if (phase == 2) {
+      // pop the next queued scheme with master > 0 (master-0 schemes are not expanded)
+      while (qh < qt && (Qq[qh] >> 24) == 0) ++qh;
+      if (qh == qt) {
+        phase = 4;  // queue exhausted: finish below
+      } else {
+        const uint32_t e = Qq[qh++];
+        const int u = (int)(e & 0xffffffu), i = (int)(e >> 24);
+        parentM = i;
+        for (int x = 1; x <= p - 1; ++x) cand[x] = Qc[(size_t)u * P + (x - 1)];
+        // child q of u (reading Q17)
+        bool valid = cand[i + 1] - cand[i] >= 2;
+        if (valid) {
+          if (q <= 1) {
+            cand[i] += 1;  // first block of stage i -> stage i-1
+            if (q == 1) {
+              if (i - 1 < 1) {
+                valid = false;
+              } else {
+                int before[33];
+                for (int x = 1; x < i - 1; ++x) before[x] = cand[x];
+                alg1_prefix(s_arg, P1, cand[i - 1], i - 1, cand);
+                bool diff = false;
+                for (int x = 1; x < i - 1; ++x) diff = diff || (cand[x] != before[x]);
+                valid = diff;
+              }
+            }
+          } else if (i > p - 2) {
+            valid = false;
+          } else {
+            cand[i + 1] -= 1;  // last block of stage i -> stage i+1
+            if (q == 3) {
+              int before[33];
+              for (int x = 1; x < i; ++x) before[x] = cand[x];
+              alg1_prefix(s_arg, P1, cand[i], i, cand);
+              bool diff = false;
+              for (int x = 1; x < i; ++x) diff = diff || (cand[x] != before[x]);
+              valid = diff;
+            }
+          }
+        }
+        // already evaluated?
+        bool dup = false;
+        if (valid) {
+          const uint32_t h = cut_hash(cand, p);
+          for (int j = 0; j < nv && !dup; ++j) {
+            if (Qh[j] != h) continue;
+            bool same = true;
+            for (int x = 1; x <= p - 1; ++x) same = same && (Qc[(size_t)j * P + (x - 1)] == cand[x]);
+            dup = same;
+          }
+        }
+        const bool isnew = valid && !dup;
+        const unsigned bal = (__ballot_sync(qmask, isnew) >> qb) & 0xFu;
+        const int cnt = __popc(bal), pre = __popc(bal & ((1u << q) - 1u));
+        const int room = vmax - nv;
+        if (cnt > room) trunc = true;
+        want = isnew && pre < room;
+        slot = nv + pre;
+      }
+    }
+
+    // ---- simulate (converged across the quads of the warp)
+    int64_t Tc = INT64_MAX;
+    int Mc = 0;
+    if (want) {
+      int cc[P + 1];
+#pragma unroll
+      for (int x = 0; x <= P; ++x) cc[x] = (x <= p) ? cand[x] : n;
+      int64_t F[P], B[P], C[P];
+      stage_costs<P>(T, p, cc, F, B, C);
+      uint32_t pb[P];
+#pragma unroll
+      for (int x = 0; x < P; ++x) pb[x] = 0;
+      Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
+      int len;
+      Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+      for (int x = 1; x <= p - 1; ++x) Qc[(size_t)slot * P + (x - 1)] = (int16_t)cand[x];
+      Qh[slot] = cut_hash(cand, p);
+    }
+
+    // ---- bookkeeping (quad-uniform)
+    if (phase == 1) {
+      Tc = __shfl_sync(qmask, Tc, qb);
+      Mc = __shfl_sync(qmask, Mc, qb);
+      if (q == 0) Qq[0] = (uint32_t)Mc << 24;
+      bestT = Tc;
+      bestNode = 0;
+      nv = 1;
+      qh = 0;
+      qt = 1;
+      nsims += (q == 0);
+      phase = 2;
+    } else if (phase == 2) {
+      const bool qual = want && Mc <= parentM;
+      const unsigned bq = (__ballot_sync(qmask, qual) >> qb) & 0xFu;
+      if (qual) Qq[qt + __popc(bq & ((1u << q) - 1u))] = (uint32_t)slot | ((uint32_t)Mc << 24);
+      // least (T, evaluation order) of this round, then against the restart's best
+      int64_t bt = Tc;
+      int bn = want ? slot : INT32_MAX;
+#pragma unroll
+      for (int o = 1; o <= 2; o <<= 1) {
+        const int64_t ot = __shfl_xor_sync(qmask, bt, o);
+        const int on = __shfl_xor_sync(qmask, bn, o);
+        if (ot < bt || (ot == bt && on < bn)) {
+          bt = ot;
+          bn = on;
+        }
+      }
+      if (bt < bestT) {
+        bestT = bt;
+        bestNode = bn;
+      }
+      const int kept = __popc((__ballot_sync(qmask, want) >> qb) & 0xFu);
+      nsims += (q == 0) ? (unsigned long long)kept : 0ull;
+      nv += kept;
+      qt += __popc(bq);
+      if (trunc) phase = 4;
+    }
+    if (phase == 4) {  // restart finished: queue exhausted or vmax reached
+      if (q == 0) {
+        if (bestT < (1ll << 43)) lane_key = min(lane_key, ((unsigned long long)bestT << 20) | r);
+        ntrunc += trunc ? 1 : 0;
+        if (A.replay)
+          for (int x = 1; x <= p - 1; ++x) A.replay[x - 1] = Qc[(size_t)bestNode * P + (x - 1)];
+      }
+      phase = 0;
+    }
+    __syncwarp();
+  }
+  if (A.stats) {
+    unsigned long long s = nsims, t = ntrunc;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) {
+      s += __shfl_xor_sync(0xffffffffu, s, o);
+      t += __shfl_xor_sync(0xffffffffu, t, o);
+    }
+    if (lane == 0) {
+      atomicAdd(&A.stats[0], s);
+      if (t) atomicAdd(&A.stats[1], t);
+    }
+  }
+  block_min_atomic(lane_key, A.key);
+}
+
+// ===========================================================================
 // Critical path with times (single candidate; thread 0).
 struct CpathArgs {
   DevTables t;
@@ -1630,6 +1881,96 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
     case 8: return heur_P<8, false>(B, s, dev, 128);
     default: return heur_P<16, false>(B, s, dev, 128);
   }
+}
+
+template <int P>
+static cudaError_t reach_P(ReachArgs* A, cudaStream_t s, int dev, uint64_t R, bool launch,
+                           int* blocks_out) {
+  const int threads = 128;
+  const int rows = A->m + min(A->p - 1, A->m);
+  const size_t narg = (size_t)(A->t.n + 1) * (A->p + 1);
+  const size_t base = ((tables_smem_bytes(A->t.npad, A->t.n) + 15) & ~size_t(15)) +
+                      ((narg + 7) & ~size_t(7)) * 2 + 32 * 4;
+  const size_t smem = base + (size_t)rows * BitsLayout<P>::WPR * 4 * threads;
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  cudaError_t e = set_smem((const void*)k_reach<P>, smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_reach<P>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  uint64_t blocks = (uint64_t)num_sms(dev) * occ;
+  const uint64_t need = (R * 4 + threads - 1) / threads;
+  if (blocks > need) blocks = need;
+  if (blocks < 1) blocks = 1;
+  *blocks_out = (int)blocks;
+  if (!launch) return cudaSuccess;
+  k_reach<P><<<(unsigned)blocks, threads, smem, s>>>(*A);
+  return cudaGetLastError();
+}
+
+static cudaError_t reach_dispatch(ReachArgs* A, cudaStream_t s, int dev, uint64_t R, bool launch,
+                                  int* blocks) {
+  switch (pick_P(A->p)) {
+    case 2: return reach_P<2>(A, s, dev, R, launch, blocks);
+    case 4: return reach_P<4>(A, s, dev, R, launch, blocks);
+    case 8: return reach_P<8>(A, s, dev, R, launch, blocks);
+    case 16: return reach_P<16>(A, s, dev, R, launch, blocks);
+    default: return reach_P<32>(A, s, dev, R, launch, blocks);
+  }
+}
+
+cudaError_t reach_scratch_bytes(const DevTables& t, int p, int m, uint32_t R, int vmax,
+                                size_t* bytes) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  ReachArgs A{};
+  A.t = t;
+  A.p = p;
+  A.m = m;
+  int blocks = 0;
+  cudaError_t e = reach_dispatch(&A, nullptr, dev, R, false, &blocks);
+  if (e != cudaSuccess) return e;
+  const size_t quads = (size_t)blocks * 32;
+  const size_t P = (size_t)pick_P(p);
+  *bytes = quads * (size_t)vmax * (P * 2 + 8) + 256;
+  return cudaSuccess;
+}
+
+cudaError_t launch_reach(const DevTables& t, int p, int m, uint64_t seed, int radius,
+                         uint32_t r_lo, uint32_t r_hi, int vmax, const int16_t* arg,
+                         const int32_t* alg1_cuts, unsigned int* counter,
+                         unsigned long long* key, unsigned long long* stats, int32_t* replay,
+                         void* scratch, cudaStream_t s) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  ReachArgs A{};
+  A.t = t;
+  A.p = p;
+  A.m = m;
+  A.seed = seed;
+  A.radius = radius;
+  A.r_lo = r_lo;
+  A.r_hi = r_hi;
+  A.arg = arg;
+  A.alg1 = alg1_cuts;
+  A.counter = counter;
+  A.key = key;
+  A.vmax = vmax;
+  A.stats = stats;
+  A.replay = replay;
+  int blocks = 0;
+  cudaError_t e = reach_dispatch(&A, s, dev, r_hi - r_lo, false, &blocks);
+  if (e != cudaSuccess) return e;
+  const size_t quads = (size_t)blocks * 32;
+  const size_t P = (size_t)pick_P(p);
+  unsigned char* b = reinterpret_cast<unsigned char*>(scratch);
+  A.g_cuts = reinterpret_cast<int16_t*>(b);
+  b += quads * (size_t)vmax * P * 2;
+  A.g_hash = reinterpret_cast<uint32_t*>(b);
+  b += quads * (size_t)vmax * 4;
+  A.g_queue = reinterpret_cast<uint32_t*>(b);
+  return reach_dispatch(&A, s, dev, r_hi - r_lo, true, &blocks);
 }
 
 size_t cpath_scratch_bytes(int p, int m) {

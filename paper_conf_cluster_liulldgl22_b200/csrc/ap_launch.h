@@ -81,6 +81,18 @@ cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t*
 // key = INT64_MAX (and counter[0..2] = 0 if non-null); precedes launch_sweep/heuristic.
 cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s);
 
+// Reachable-set search (NEXT N1): restarts [r_lo, r_hi), key = min (T << 20 | r).
+// scratch: reach_scratch_bytes() for the same (p, m, R = r_hi - r_lo, vmax); counter[0]
+// zeroed (launch_init_key); stats (u64[2]: sims, truncated restarts) zeroed or NULL;
+// replay (int32[p-1]) non-null: the single restart r_lo's best cut vector.
+cudaError_t reach_scratch_bytes(const DevTables& t, int p, int m, uint32_t R, int vmax,
+                                size_t* bytes);
+cudaError_t launch_reach(const DevTables& t, int p, int m, uint64_t seed, int radius,
+                         uint32_t r_lo, uint32_t r_hi, int vmax, const int16_t* arg,
+                         const int32_t* alg1_cuts, unsigned int* counter,
+                         unsigned long long* key, unsigned long long* stats, int32_t* replay,
+                         void* scratch, cudaStream_t s);
+
 // Decode helper: unrank lex rank -> cut vector int32[p-1].
 cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,
                           cudaStream_t s);

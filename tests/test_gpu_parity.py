@@ -688,3 +688,66 @@ def test_two_phase_configs_match_packed(ap, cfg):
     key = _search(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
     T, idx = _search2(ap, plan, wl.p, wl.m, wl.k_lo, wl.k_hi)
     assert key == (T << rank_bits(N, K)) | idx
+
+
+# --------------------------------------------------------------------------- N1 reach
+def _reach(ap, plan, p, m, seed, radius, r_lo, r_hi, vmax):
+    import torch
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    ap.ap_search_reachable(plan, p, m, seed, radius, r_lo, r_hi, vmax, key)
+    torch.cuda.synchronize()
+    return int(key.item()), ap.ap_last_sims(), ap.ap_last_truncated()
+
+
+def test_reach_random_vs_oracle(ap, oracle_mod):
+    """ap_search_reachable == oracle or_reach: winner (T, restart), decoded cuts, total
+    simulations and truncated-restart count -- including tiny vmax (truncation)."""
+    rng = np.random.default_rng(31)
+    for trial in range(16):
+        kind = ["uniform", "b3f", "small", "equal"][trial % 4]
+        n = int(rng.integers(4, 60))
+        f, b, a = synth.random_tables(500 + trial, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p = int(rng.integers(1, min(n, 20) + 1))
+        m = int(rng.choice([1, 2, p, p + 3, 24]))
+        seed, radius = int(rng.integers(0, 1 << 30)), int(rng.integers(0, 4))
+        R = int(rng.integers(1, 200))
+        vmax = int(rng.choice([1, 3, 8, 1024]))
+        key, sims, trunc = _reach(ap, plan, p, m, seed, radius, 0, R, vmax)
+        o = M.reach(p, m, seed, radius, 0, R, vmax=vmax)
+        assert (key >> 20, key & 0xFFFFF) == (o["T"], o["restart"]), (trial, n, p, m, vmax)
+        assert (sims, trunc) == (o["sims"], o["truncated"]), (trial, n, p, m, vmax)
+        res = ap.ap_decode_reachable(plan, p, m, seed, radius, vmax, key)
+        assert res["time_ns"] == o["T"] and res["cuts"] == [int(x) for x in o["cuts"]]
+        assert res["master"] == M.simulate(p, m, o["cuts"])["master"]
+
+
+@pytest.mark.parametrize("cfg,R", [(2, 1024), (3, 512), (4, 256), (5, 2048)])
+def test_reach_configs_vs_oracle(ap, oracle_mod, cfg, R):
+    """Configs: same winner, simulations and truncations as the oracle, and never
+    worse than the greedy walk over the same restarts."""
+    wl = synth.config(cfg)
+    f, b, a = wl.arrays()
+    M = oracle_mod.Model.from_workload(wl)
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    key, sims, trunc = _reach(ap, plan, wl.p, wl.m, wl.seed, wl.radius, 0, R, 1024)
+    o = M.reach_parallel(wl.p, wl.m, wl.seed, wl.radius, 0, R, vmax=1024)
+    assert (key >> 20, key & 0xFFFFF, sims, trunc) == (o["T"], o["restart"], o["sims"], o["truncated"])
+    import torch
+    hk = torch.empty(1, dtype=torch.int64, device="cuda")
+    ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, R, 0, hk)
+    torch.cuda.synchronize()
+    assert key >> 20 <= int(hk.item()) >> 20
+
+
+def test_reach_errors(ap):
+    import torch
+    f, b, a = synth.random_tables(3, 10, "uniform")
+    plan = _plan(ap, f, b, a, synth.link_for("uniform"))
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    for args in [(3, 4, 0, 2, 5, 5, 8), (3, 4, 0, 2, 0, 8, 0), (3, 4, 0, -1, 0, 8, 8),
+                 (3, 4, 0, 2, 0, (1 << 20) + 1, 8)]:
+        with pytest.raises(ap.APError):
+            ap.ap_search_reachable(plan, *args, key)

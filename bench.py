@@ -477,6 +477,37 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
                  "sims_per_s": float(sims5[0]) / (float(t[0]) / 1e3),
                  "time_to_plan_ms": float(t[0]), "T_ns": r5["time_ns"], "restart": r5["restart"],
                  "cuts": r5["cuts"], "slicer_T_ns": [int(x) for x in Tk], "slicer_best_k": bk}
+    # certified bound (NEXT N3): T* >= minLB, so the plan is within `certified_gap` of optimal
+    lb, _ = ap.ap_min_lower_bound(plan5, wl.p, wl.m, 1)
+    out["C5"]["certified_minlb_ns"] = lb
+    out["C5"]["certified_gap"] = (r5["time_ns"] - lb) / lb
+
+    # reachable-set search (NEXT N1) over the same restarts
+    vmax = 1024
+
+    def s5r():
+        ap.ap_search_reachable(plan5, wl.p, wl.m, wl.seed, wl.radius, rlo, rhi, vmax, key)
+        if world > 1:
+            dist.all_reduce(key, op=dist.ReduceOp.MIN)
+        return ap.ap_decode_reachable(plan5, wl.p, wl.m, wl.seed, wl.radius, vmax, int(key.item()))
+    s5r()
+    times = []
+    for _ in range(3):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(); rr = s5r(); e1.record(); torch.cuda.synchronize()
+        times.append(e0.elapsed_time(e1))
+    t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
+    st = torch.tensor([float(ap.ap_last_sims()), float(ap.ap_last_truncated())],
+                      dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(st, op=dist.ReduceOp.SUM)
+    out["C5_reachable"] = {"workload": wl.name + "-reachable-set", "restarts": wl.restarts,
+                           "vmax": vmax, "time_to_plan_ms": float(t[0]),
+                           "sims_per_step": int(st[0]), "truncated_restarts": int(st[1]),
+                           "sims_per_s": float(st[0]) / (float(t[0]) / 1e3),
+                           "T_ns": rr["time_ns"], "restart": rr["restart"]}
     return out
 
 

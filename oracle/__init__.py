@@ -65,6 +65,12 @@ def _load():
             lib.or_alg1_reconstruct.argtypes = [P(i32), i32, i32, i32, i32, P(i32)]
             lib.or_min_lb.restype = i32
             lib.or_min_lb.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, i32, P(i64), P(i32)]
+            lib.or_stage_feasible.restype = i32
+            lib.or_stage_feasible.argtypes = [i32, P(i64), P(i64), i64, i32, i32, P(i32)]
+            lib.or_exhaustive_mem.restype = i32
+            lib.or_exhaustive_mem.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, i32, i32,
+                                              P(i64), P(i64), i64, P(i64), P(u64), P(i32),
+                                              P(i32), P(u64)]
             lib.or_count.restype = u64
             lib.or_count.argtypes = [i32, i32]
             lib.or_rank.restype = u64
@@ -223,6 +229,46 @@ class Model:
         best = dict(best)
         best["sims"] = sum(d["sims"] for d in res)
         return best
+
+    # ------------------------------------------------- N4 depth + memory (R-N4)
+    def feasible(self, p, m, cuts, static_bytes, stash_bytes, cap) -> bool:
+        lib = _load()
+        c = _i32(cuts) if p > 1 else np.zeros(1, np.int32)
+        return bool(lib.or_stage_feasible(self.n, _p(_i64(static_bytes), C.c_int64),
+                                          _p(_i64(stash_bytes), C.c_int64), int(cap), p, m,
+                                          _p(c, C.c_int32)))
+
+    def exhaustive_mem(self, p, m, k_lo, k_hi, static_bytes, stash_bytes, cap):
+        """Exhaustive argmin over the memory-feasible partitions; T = None if none."""
+        lib = _load()
+        T = C.c_int64(); r = C.c_uint64(); k = C.c_int32(); sims = C.c_uint64()
+        cuts = np.zeros(max(p - 1, 1), np.int32)
+        sb, tb = _i64(static_bytes), _i64(stash_bytes)
+        _chk(lib.or_exhaustive_mem(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                                   _p(self.comm, C.c_int64), p, m, k_lo, k_hi,
+                                   _p(sb, C.c_int64), _p(tb, C.c_int64), int(cap),
+                                   C.byref(T), C.byref(r), C.byref(k), _p(cuts, C.c_int32),
+                                   C.byref(sims)))
+        if T.value == (1 << 63) - 1:
+            return {"T": None, "sims": sims.value}
+        return {"T": T.value, "rank": r.value, "k": k.value, "cuts": cuts[: p - 1].copy(),
+                "sims": sims.value}
+
+    def plan_depths(self, n_gpus, microbatches, static_bytes, stash_bytes, cap, k_lo=1, k_hi=1):
+        """Outer planner loop (NEXT N4, reading R-N4): every depth p dividing n_gpus
+        (p <= n) whose data-parallel width dp = n_gpus/p divides `microbatches`;
+        m = microbatches/dp; the feasible argmin per p; best = least (T, p)."""
+        per = []
+        for p in range(1, min(self.n, n_gpus) + 1):
+            if n_gpus % p or microbatches % (n_gpus // p):
+                continue
+            m = microbatches // (n_gpus // p)
+            r = self.exhaustive_mem(p, m, k_lo, k_hi, static_bytes, stash_bytes, cap)
+            r.update({"p": p, "m": m, "dp": n_gpus // p})
+            per.append(r)
+        feas = [r for r in per if r["T"] is not None]
+        best = min(feas, key=lambda r: (r["T"], r["p"])) if feas else None
+        return best, per
 
     def lower_bound(self, p, m, K, cuts) -> int:
         lib = _load()

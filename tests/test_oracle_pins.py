@@ -799,3 +799,71 @@ def test_reach_truncation_and_bounds(oracle_mod):
     wl = synth.config(2)
     M = oracle_mod.Model.from_workload(wl)
     assert M.reach_restart(wl.p, wl.m, wl.seed, wl.radius, 0)["T"] == 89891590
+
+
+# ----------------------------------------------------------------------------- N4 memory
+def test_N4_inflight_count_matches_the_schedule(oracle_mod):
+    """Reading R-N4's in-flight count: the most micro-batches stage x holds between
+    their FP and BP, read off the oracle's own 1F1B op order (ops sorted by start on
+    each stage, positive costs), is min(p - x, m)."""
+    for p in range(1, 7):
+        for m in range(1, 10):
+            n = p + 2
+            M = oracle_mod.Model([3 + i for i in range(n)], [5 + 2 * i for i in range(n)],
+                                 [7] * n, 10**9)
+            cuts = list(range(1, p))
+            ops = M.simulate(p, m, cuts, want_all=True)["ops"]
+            for x in range(p):
+                seq = sorted((o[4], o[1]) for o in ops if o[0] == x)
+                cur = most = 0
+                for _, kind in seq:
+                    cur += 1 if kind == 0 else -1
+                    most = max(most, cur)
+                assert most == min(p - x, m), (p, m, x)
+
+
+def test_N4_memory_feasibility_handworked(oracle_mod):
+    """n = 4, p = 2, m = 3, static 10 B and stash 1 B per sub-layer: in-flight 2 on
+    stage 0 and 1 on stage 1, so cut 1 needs (12, 33) B, cut 2 (24, 22) B, cut 3
+    (36, 11) B.  cap 33 admits cuts 1 and 2, cap 24 only cut 2, cap 23 none."""
+    M = oracle_mod.Model([4, 1, 1, 4], [8, 2, 2, 8], [0, 0, 0, 0], 10**9)
+    st, sh = [10] * 4, [1] * 4
+    assert [M.feasible(2, 3, [c], st, sh, 33) for c in (1, 2, 3)] == [True, True, False]
+    assert [M.feasible(2, 3, [c], st, sh, 24) for c in (1, 2, 3)] == [False, True, False]
+    assert not any(M.feasible(2, 3, [c], st, sh, 23) for c in (1, 2, 3))
+    r = M.exhaustive_mem(2, 3, 1, 1, st, sh, 33)
+    Ts = {c: M.T(2, 3, [c]) for c in (1, 2)}
+    assert r["T"] == min(Ts.values()) and list(r["cuts"]) == [min(Ts, key=lambda c: (Ts[c], c))]
+    assert M.exhaustive_mem(2, 3, 1, 1, st, sh, 24)["cuts"][0] == 2
+    assert M.exhaustive_mem(2, 3, 1, 1, st, sh, 23)["T"] is None
+
+
+def test_N4_plan_depths_properties(oracle_mod):
+    """Unlimited memory: every depth's feasible argmin is the plain exhaustive one, and
+    the outer loop picks p = 1 with T = m*sum(f+b) (P4; a deeper pipeline only adds
+    fill and drain).  Shrinking the capacity never lowers the chosen T, and below the
+    smallest possible stage footprint nothing is feasible."""
+    for seed in range(12):
+        kind = ["uniform", "b3f", "small"][seed % 3]
+        n = 6 + seed % 6
+        f, b, a = synth.random_tables(seed, n, kind)
+        M = oracle_mod.Model(f, b, a, synth.link_for(kind))
+        rng = np.random.default_rng(seed)
+        st = rng.integers(1, 1000, n)
+        sh = rng.integers(0, 100, n)
+        G, mb = 4, 8
+        best, per = M.plan_depths(G, mb, st, sh, 1 << 60)
+        for r in per:
+            ex = M.exhaustive(r["p"], r["m"])
+            assert (r["T"], r["rank"]) == (ex["T"], ex["rank"])
+        assert best["p"] == 1 and best["T"] == (mb // G) * int(f.sum() + b.sum())
+        prevT = best["T"]
+        for cap in sorted({int(st.sum() + 8 * sh.sum()) // d for d in (1, 2, 3, 4, 6, 8)},
+                          reverse=True):
+            bst, _ = M.plan_depths(G, mb, st, sh, cap)
+            if bst is None:
+                prevT = None
+                continue
+            assert prevT is not None and bst["T"] >= prevT
+            prevT = bst["T"]
+        assert M.plan_depths(G, mb, st, sh, int(st.min()) - 1)[0] is None

@@ -508,6 +508,28 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
                            "sims_per_step": int(st[0]), "truncated_restarts": int(st[1]),
                            "sims_per_s": float(st[0]) / (float(t[0]) / 1e3),
                            "T_ns": rr["time_ns"], "restart": rr["restart"]}
+
+    # outer loop over pipeline depth with the memory model (NEXT N4)
+    from paper_conf_cluster_liulldgl22_b200.search import plan_pipeline_depth
+    dw = synth.depth_config()
+    f, b, a = dw.base.arrays()
+    plan4 = ap.ap_plan_create(f, b, a, dw.base.link_bytes_per_s, device=dev.index)
+    ap.ap_plan_set_memory(plan4, dw.static_bytes, dw.stash_bytes, dw.cap_bytes)
+    plan_pipeline_depth(plan4, dw.n_gpus, dw.microbatches)
+    times = []
+    for _ in range(3):
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(); r4 = plan_pipeline_depth(plan4, dw.n_gpus, dw.microbatches); e1.record()
+        torch.cuda.synchronize()
+        times.append(e0.elapsed_time(e1))
+    t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    out["N4_depth"] = {"workload": dw.name, "time_to_plan_ms": float(t[0]),
+                       "sims_per_step": sum(r["sims"] for r in r4["per_depth"]),
+                       "best": {k: r4["best"][k] for k in ("p", "dp", "m", "T", "cuts")},
+                       "per_depth_T_ns": {r["p"]: r["T"] for r in r4["per_depth"]}}
     return out
 
 

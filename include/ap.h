@@ -92,6 +92,20 @@ void ap_plan_destroy(ap_plan* plan);
 /* Number of sub-layers and comm_ns table (host copy) of a plan.  comm may be NULL. */
 ap_status ap_plan_info(const ap_plan* plan, int32_t* n, int64_t* comm_ns);
 
+/*
+ * ap_plan_set_memory -- attach the memory model of NEXT N4 (reading R-N4) to
+ * a plan, for AP_SEARCH_MEMORY searches and the outer loop over pipeline depth.
+ *   static_bytes  host int64[n] >= 0: bytes a sub-layer holds for the whole iteration
+ *                 on its stage (weights, gradients, optimizer state).
+ *   stash_bytes   host int64[n] >= 0: bytes it keeps per in-flight micro-batch between
+ *                 FP and BP (with activation checkpointing: its input).
+ *   cap_bytes     per-GPU capacity available to these two terms.
+ * Replaces a previous model.  Not synchronised with searches running on the plan.
+ * Errors: INVALID (NULL, negative), RANGE (sum(static) + 32*sum(stash) >= 2^62), NOMEM.
+ */
+ap_status ap_plan_set_memory(ap_plan* plan, const int64_t* static_bytes,
+                             const int64_t* stash_bytes, int64_t cap_bytes);
+
 /* C(n-1, p-1): the size of the partition space.  RANGE when it
  * is >= 2^63.  INVALID unless 1 <= p <= n. */
 ap_status ap_count(int32_t n, int32_t p, uint64_t* out);
@@ -158,6 +172,14 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
 #define AP_SEARCH_FULL 0
 #define AP_SEARCH_KFACTOR 1
 #define AP_SEARCH_PRUNED 2
+/* AP_SEARCH_MEMORY (NEXT N4; reading R-N4): the full sweep restricted to the
+ * partitions that fit the plan's memory model (ap_plan_set_memory; INVALID without it):
+ * every stage x must satisfy  sum(static) + min(p-x, m) * sum(stash) <= cap  over its
+ * sub-layers (min(p-x, m) = the micro-batches 1F1B keeps in flight on stage x).  Runs
+ * on the generic exact kernel.  T_ref is the Alg.-1 partition's T when that partition
+ * fits, else the overflow guard's bound on any T (then the packed key usually does not
+ * fit and ap_search_exhaustive2 applies).  INT64_MAX when nothing fits. */
+#define AP_SEARCH_MEMORY 4
 ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
                                     int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
                                     int32_t mode, int64_t* key, ap_stream_t stream);

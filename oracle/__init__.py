@@ -69,8 +69,8 @@ def _load():
             lib.or_stage_feasible.argtypes = [i32, P(i64), P(i64), i64, i32, i32, P(i32)]
             lib.or_exhaustive_mem.restype = i32
             lib.or_exhaustive_mem.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, i32, i32,
-                                              P(i64), P(i64), i64, P(i64), P(u64), P(i32),
-                                              P(i32), P(u64)]
+                                              P(i64), P(i64), i64, u64, u64, P(i64), P(u64),
+                                              P(i32), P(i32), P(u64)]
             lib.or_count.restype = u64
             lib.or_count.argtypes = [i32, i32]
             lib.or_rank.restype = u64
@@ -238,16 +238,19 @@ class Model:
                                           _p(_i64(stash_bytes), C.c_int64), int(cap), p, m,
                                           _p(c, C.c_int32)))
 
-    def exhaustive_mem(self, p, m, k_lo, k_hi, static_bytes, stash_bytes, cap):
+    def exhaustive_mem(self, p, m, k_lo, k_hi, static_bytes, stash_bytes, cap, rank_lo=0,
+                       rank_hi=None):
         """Exhaustive argmin over the memory-feasible partitions; T = None if none."""
         lib = _load()
+        if rank_hi is None:
+            rank_hi = count(self.n, p)
         T = C.c_int64(); r = C.c_uint64(); k = C.c_int32(); sims = C.c_uint64()
         cuts = np.zeros(max(p - 1, 1), np.int32)
         sb, tb = _i64(static_bytes), _i64(stash_bytes)
         _chk(lib.or_exhaustive_mem(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
                                    _p(self.comm, C.c_int64), p, m, k_lo, k_hi,
                                    _p(sb, C.c_int64), _p(tb, C.c_int64), int(cap),
-                                   C.byref(T), C.byref(r), C.byref(k), _p(cuts, C.c_int32),
+                                   int(rank_lo), int(rank_hi), C.byref(T), C.byref(r), C.byref(k), _p(cuts, C.c_int32),
                                    C.byref(sims)))
         if T.value == (1 << 63) - 1:
             return {"T": None, "sims": sims.value}

@@ -100,6 +100,8 @@ def _load_lib():
     lib.ap_decode_reachable.argtypes = [vp, i32, i32, u64, i32, i32, i64, P(ApResult)]
     lib.ap_last_truncated.restype = i32
     lib.ap_last_truncated.argtypes = [P(u64)]
+    lib.ap_plan_set_memory.restype = i32
+    lib.ap_plan_set_memory.argtypes = [vp, P(i64), P(i64), i64]
     lib.ap_min_lower_bound.restype = i32
     lib.ap_min_lower_bound.argtypes = [vp, i32, i32, i32, P(i64), P(i32)]
     lib.ap_last_launch.restype = None
@@ -115,6 +117,7 @@ lib = _load_lib()
 
 # every symbol include/ap.h declares (checked by tests/test_abi.py)
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
+           "ap_plan_set_memory",
            "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_exhaustive_mode",
            "ap_search_exhaustive2", "ap_key2_select",
            "ap_search_heuristic", "ap_search_reachable", "ap_decode_reachable",
@@ -239,7 +242,7 @@ def ap_search_exhaustive(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank_
                                     _stream(stream)))
 
 
-AP_SEARCH_FULL, AP_SEARCH_KFACTOR, AP_SEARCH_PRUNED = 0, 1, 2
+AP_SEARCH_FULL, AP_SEARCH_KFACTOR, AP_SEARCH_PRUNED, AP_SEARCH_MEMORY = 0, 1, 2, 4
 
 
 def ap_search_exhaustive_mode(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank_lo: int,
@@ -356,6 +359,16 @@ def ap_alg1(plan: Plan, p: int):
     _check(lib.ap_alg1(plan.handle, int(p), cuts.ctypes.data_as(C.POINTER(C.c_int32)),
                        C.byref(v)))
     return cuts[: p - 1].copy(), v.value
+
+
+def ap_plan_set_memory(plan: Plan, static_bytes, stash_bytes, cap_bytes: int):
+    """Attach the N4 memory model (include/ap.h) for AP_SEARCH_MEMORY searches."""
+    sb = np.ascontiguousarray(static_bytes, dtype=np.int64)
+    tb = np.ascontiguousarray(stash_bytes, dtype=np.int64)
+    if sb.shape != (plan.n,) or tb.shape != (plan.n,):
+        raise ValueError("memory tables must have n entries")
+    _check(lib.ap_plan_set_memory(plan.handle, sb.ctypes.data_as(C.POINTER(C.c_int64)),
+                                  tb.ctypes.data_as(C.POINTER(C.c_int64)), int(cap_bytes)))
 
 
 def ap_min_lower_bound(plan: Plan, p: int, m: int, K: int = 1):

@@ -7,6 +7,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
+#include <algorithm>
 #include <cstring>
 #include <atomic>
 #include <mutex>
@@ -209,7 +210,20 @@ struct ap_plan {
   int64_t* d_tab = nullptr;
   uint64_t* d_binom = nullptr;
   cudaMemPool_t pool = nullptr;
+  // memory model (ap_plan_set_memory, NEXT N4): prefix sums of static and stash bytes
+  bool has_mem = false;
+  std::vector<int64_t> mem_pw, mem_ps;  // [n+1]
+  int64_t mem_cap = 0;
+  int64_t* d_mem = nullptr;  // device [2][n+1]: PW, PS
   apk::DevTables dev() const { return apk::DevTables{d_tab, d_binom, n, npad}; }
+  bool feasible(int p, int m, const int32_t* cuts) const {
+    for (int x = 0; x < p; ++x) {
+      const int lo = x == 0 ? 0 : cuts[x - 1], hi = x == p - 1 ? n : cuts[x];
+      const int64_t inflight = (p - x < m) ? p - x : m;
+      if (mem_pw[hi] - mem_pw[lo] + inflight * (mem_ps[hi] - mem_ps[lo]) > mem_cap) return false;
+    }
+    return true;
+  }
 };
 
 extern "C" {
@@ -350,10 +364,51 @@ void ap_plan_destroy(ap_plan* plan) {
     cudaStream_t s0 = nullptr;
     if (plan->d_tab && internal_stream(plan->device, &s0) == cudaSuccess) {
       cudaFreeAsync(plan->d_tab, s0);
+      if (plan->d_mem) cudaFreeAsync(plan->d_mem, s0);
       cudaStreamSynchronize(s0);
     }
   }
   delete plan;
+}
+
+ap_status ap_plan_set_memory(ap_plan* plan, const int64_t* static_bytes, const int64_t* stash_bytes,
+                             int64_t cap_bytes) {
+  g_err.clear();
+  if (!plan) return fail(AP_ERR_INVALID, "plan is NULL");
+  if (!static_bytes || !stash_bytes) return fail(AP_ERR_INVALID, "NULL table");
+  if (cap_bytes < 0) return fail(AP_ERR_INVALID, "cap_bytes < 0");
+  const int n = plan->n;
+  std::vector<int64_t> pw(n + 1, 0), ps(n + 1, 0);
+  unsigned __int128 tw = 0, ts = 0;
+  for (int i = 0; i < n; ++i) {
+    if (static_bytes[i] < 0 || stash_bytes[i] < 0)
+      return fail(AP_ERR_INVALID, "negative memory entry at sub-layer %d", i);
+    tw += (uint64_t)static_bytes[i];
+    ts += (uint64_t)stash_bytes[i];
+    pw[i + 1] = pw[i] + static_bytes[i];
+    ps[i + 1] = ps[i] + stash_bytes[i];
+  }
+  // a stage's footprint is at most sum(static) + AP_MAX_P * sum(stash)
+  if (tw + (unsigned __int128)AP_MAX_P * ts >= ((unsigned __int128)1 << 62))
+    return fail(AP_ERR_RANGE, "memory tables too large (>= 2^62 bytes)");
+  DeviceGuard g(plan->device);
+  cudaStream_t s;
+  AP_CUDA(internal_stream(plan->device, &s));
+  if (!plan->d_mem) {
+    cudaError_t e = cudaMallocFromPoolAsync((void**)&plan->d_mem, 2 * (size_t)(n + 1) * 8,
+                                            plan->pool, s);
+    if (e != cudaSuccess) return fail(AP_ERR_NOMEM, "memory tables");
+  }
+  std::vector<int64_t> both(2 * (size_t)(n + 1));
+  std::copy(pw.begin(), pw.end(), both.begin());
+  std::copy(ps.begin(), ps.end(), both.begin() + (n + 1));
+  AP_CUDA(cudaMemcpyAsync(plan->d_mem, both.data(), both.size() * 8, cudaMemcpyHostToDevice, s));
+  AP_CUDA(cudaStreamSynchronize(s));
+  plan->mem_pw = std::move(pw);
+  plan->mem_ps = std::move(ps);
+  plan->mem_cap = cap_bytes;
+  plan->has_mem = true;
+  return AP_OK;
 }
 
 ap_status ap_plan_info(const ap_plan* plan, int32_t* n, int64_t* comm_ns) {
@@ -524,11 +579,13 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
                                  int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int32_t mode,
                                  int64_t* key, int64_t* out2, ap_stream_t stream) {
   g_err.clear();
-  if (mode < AP_SEARCH_FULL || mode > AP_SEARCH_PRUNED)
+  const bool mem = (mode == AP_SEARCH_MEMORY);
+  if (!mem && (mode < AP_SEARCH_FULL || mode > AP_SEARCH_PRUNED))
     return fail(AP_ERR_INVALID, "search mode %d", mode);
   ap_status st = check_pm(plan, p, m);
   if (st != AP_OK) return st;
   if (!key && !out2) return fail(AP_ERR_INVALID, "key is NULL");
+  if (mem && !plan->has_mem) return fail(AP_ERR_INVALID, "AP_SEARCH_MEMORY without ap_plan_set_memory");
   if (k_lo < 1 || k_hi < k_lo || k_hi > AP_MAX_K)
     return fail(AP_ERR_INVALID, "k range [%d, %d] outside [1, %d]", k_lo, k_hi, AP_MAX_K);
   uint64_t N;
@@ -554,9 +611,18 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 0, 1,
                            d_tref, nullptr, s, &launches));
   int64_t tref = 0;
+  int32_t a1h[32] = {0};
   AP_CUDA(cudaMemcpyAsync(&tref, d_tref, 8, cudaMemcpyDeviceToHost, s));
+  if (mem && p > 1) AP_CUDA(cudaMemcpyAsync(a1h, d_a1, 4 * (size_t)(p - 1), cudaMemcpyDeviceToHost, s));
   AP_CUDA(cudaStreamSynchronize(s));
   if (tref < 0) return fail(AP_ERR_CUDA, "T_ref evaluation failed");
+  if (mem && !plan->feasible(p, m, a1h)) {
+    // the Alg.-1 partition does not fit: no attained feasible T to bound the search
+    // with, so every candidate stays (S = the overflow guard's bound on any T)
+    const unsigned __int128 tot = (unsigned __int128)m * (uint64_t)(plan->sum_f + plan->sum_b) +
+                                  (unsigned __int128)2 * m * (p - 1) * (uint64_t)plan->max_comm;
+    tref = (int64_t)tot;
+  }
   if (key && (rb >= 63 || (uint64_t)tref >= ((1ull << (63 - rb)) - 1)))
     return fail(AP_ERR_RANGE, "key packing: T_ref=%lld needs %d bits + %d rank bits > 63",
                 (long long)tref, bitlen((unsigned __int128)tref), rb);
@@ -589,9 +655,14 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
     AP_CUDA(sc.get((void**)&rec, 16 * (size_t)apk::sweep_max_blocks(plan->device)));
   }
   AP_CUDA(g_timer.record(0, s, plan->device));
+  if (mem) {
+    want_u32 = 0;  // memory mode: the generic exact kernel with the feasibility filter
+    force_generic = 1;
+  }
   AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, S, rb, want_u32,
-                            clamp_rows, force_generic, mode,
-                            reinterpret_cast<unsigned long long*>(key), s, &sp, rec));
+                            clamp_rows, force_generic, mem ? AP_SEARCH_FULL : mode,
+                            reinterpret_cast<unsigned long long*>(key), s, &sp, rec,
+                            mem ? plan->d_mem : nullptr, plan->mem_cap));
   if (rec) {
     AP_CUDA(apk::launch_reduce2(rec, sp.blocks, reinterpret_cast<long long*>(out2), s));
     ++launches;

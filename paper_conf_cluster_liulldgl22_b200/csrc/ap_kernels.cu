@@ -257,6 +257,8 @@ struct SweepArgs {
   uint32_t one;    // = 1 (adds are plain operators; kept for the XOps interface)
   int mode;        // 0 full, 1 k-factored, 2 k-factored + lower-bound skipping
   unsigned long long* rec;  // two-phase: per-CTA (T, index) records instead of `key`
+  const int64_t* mem;       // memory filter (generic kernel): [2][n+1] prefix sums
+  int64_t mem_cap;
 };
 
 AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
@@ -528,6 +530,13 @@ __global__ void __launch_bounds__(128) k_sweep_generic(SweepArgs A) {
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
   const int n = A.t.n, p = A.p, m = A.m;
+  const int64_t* s_mem = nullptr;
+  if (A.mem) {
+    int64_t* sm = reinterpret_cast<int64_t*>(smem + ((used + 15) & ~size_t(15)));
+    for (int i = threadIdx.x; i < 2 * (n + 1); i += blockDim.x) sm[i] = A.mem[i];
+    __syncthreads();
+    s_mem = sm;
+  }
   const uint64_t K = (uint64_t)(A.k_hi - A.k_lo + 1);
   int64_t bestT = (int64_t)A.S;
   uint64_t bestIdx = 0;
@@ -566,7 +575,20 @@ __global__ void __launch_bounds__(128) k_sweep_generic(SweepArgs A) {
     for (uint64_t r = r0; r < r1; ++r) {
       int64_t F[P], B[P], C[P];
       stage_costs<P>(T, p, c, F, B, C);
-      for (int k = A.k_lo; k <= A.k_hi; ++k) {
+      bool fits = true;
+      if (s_mem) {
+        // reading R-N4: static bytes + min(p-x, m) stashed micro-batches per stage
+#pragma unroll
+        for (int x = 0; x < P; ++x) {
+          if (x < p) {
+            const int64_t inflight = (p - x < m) ? p - x : m;
+            const int64_t need = (s_mem[c[x + 1]] - s_mem[c[x]]) +
+                                 inflight * (s_mem[n + 1 + c[x + 1]] - s_mem[n + 1 + c[x]]);
+            fits = fits && need <= A.mem_cap;
+          }
+        }
+      }
+      for (int k = A.k_lo; fits && k <= A.k_hi; ++k) {
         const int64_t Tc = sim_exact<P, 0>(p, m, k, F, B, C, nob, pb, not_);
         if (Tc < bestT) {
           bestT = Tc;
@@ -1733,7 +1755,8 @@ static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int
 
 template <int P>
 static cudaError_t sweep_generic_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int dev) {
-  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n);
+  const size_t smem = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
+                      (A.mem ? 2 * (size_t)(A.t.n + 1) * 8 : 0);
   const void* fn = (const void*)k_sweep_generic<P>;
   cudaError_t e = set_smem(fn, smem);
   if (e != cudaSuccess) return e;
@@ -1800,11 +1823,13 @@ bool has_exact(int p) {
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
-                         SweepPlan* sp, unsigned long long* rec) {
+                         SweepPlan* sp, unsigned long long* rec, const int64_t* mem,
+                         int64_t mem_cap) {
   int dev = 0;
   cudaGetDevice(&dev);
-  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u, mode, rec};
-  const bool exact = has_exact(p) && m >= p && (!force_generic || mode != 0);
+  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u, mode, rec,
+              mem, mem_cap};
+  const bool exact = !mem && has_exact(p) && m >= p && (!force_generic || mode != 0);
   sp->exact_p = exact ? 1 : 0;
   sp->fast_u32 = (exact && want_u32) ? 1 : 0;
   if (exact) return sweep_exact_dispatch(p, sp->fast_u32, A, s, sp, dev);

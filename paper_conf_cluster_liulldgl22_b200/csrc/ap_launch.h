@@ -43,7 +43,8 @@ struct SweepPlan {
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
-                         SweepPlan* plan_out, unsigned long long* rec = nullptr);
+                         SweepPlan* plan_out, unsigned long long* rec = nullptr,
+                         const int64_t* mem = nullptr, int64_t mem_cap = 0);
 
 // Two-phase reduction (NEXT N3).  With `rec` (u64[2 * sweep_max_blocks(dev)]) passed
 // to launch_sweep, each CTA stores its lexicographic min (T, index) there instead of

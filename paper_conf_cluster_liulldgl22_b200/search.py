@@ -15,7 +15,7 @@ from typing import Optional
 
 import torch
 
-from . import (AP_ERR_RANGE, INT64_MAX, APError, Plan, ap_count, ap_decode,
+from . import (AP_ERR_RANGE, AP_SEARCH_MEMORY, INT64_MAX, APError, Plan, ap_count, ap_decode,
                ap_key2_select, ap_search_exhaustive, ap_search_exhaustive2,
                ap_search_heuristic)
 
@@ -110,7 +110,7 @@ def search_exhaustive(plan: Plan, p: int, m: int, k_lo: int = 1, k_hi: int = 1,
         min_allreduce_key(key, dist, group)
         kv = int(key.item())
         out["key"] = kv
-        if decode:
+        if decode and kv != INT64_MAX:
             out.update(ap_decode(plan, 0, p, m, k_lo, k_hi, key=kv))
         return out
     local = torch.empty(2, dtype=torch.int64, device=dev)
@@ -126,6 +126,37 @@ def search_exhaustive(plan: Plan, p: int, m: int, k_lo: int = 1, k_hi: int = 1,
             raise RuntimeError(f"two-phase decode: T*={T}, re-simulated {res['time_ns']}")
         out.update(res)
     return out
+
+
+def plan_pipeline_depth(plan: Plan, n_gpus: int, microbatches: int, k_lo: int = 1,
+                        k_hi: int = 1, group=None) -> dict:
+    """NEXT N4 (reading R-N4): the outer planner loop over pipeline depth.
+    Needs ap_plan_set_memory on `plan`.  For every depth p dividing n_gpus (p <= n,
+    <= AP_MAX_P) whose data-parallel width dp = n_gpus / p divides `microbatches`:
+    m = microbatches / dp, and the exact argmin over the memory-feasible partitions
+    (AP_SEARCH_MEMORY, sharded over the ranks like search_exhaustive).  The plan is the
+    least (T, p); no data-parallel all-reduce term (reading Q12)."""
+    from . import AP_MAX_P
+    per = []
+    for p in range(1, min(plan.n, n_gpus, AP_MAX_P) + 1):
+        if n_gpus % p or microbatches % (n_gpus // p):
+            continue
+        m = microbatches // (n_gpus // p)
+        r = search_exhaustive(plan, p, m, k_lo, k_hi, group=group, decode=False,
+                              mode=AP_SEARCH_MEMORY)
+        row = {"p": p, "dp": n_gpus // p, "m": m, "two_phase": r["two_phase"],
+               "sims": r["total_sims"]}
+        key = r["key"]
+        if key == INT64_MAX:
+            row["T"] = None
+        else:
+            res = ap_decode(plan, 2 if r["two_phase"] else 0, p, m, k_lo, k_hi, key=key)
+            row.update({"T": res["time_ns"], "rank": res["rank"], "k": res["k"],
+                        "cuts": res["cuts"], "master": res["master"]})
+        per.append(row)
+    feas = [r for r in per if r["T"] is not None]
+    best = min(feas, key=lambda r: (r["T"], r["p"])) if feas else None
+    return {"best": best, "per_depth": per}
 
 
 def search_heuristic(plan: Plan, p: int, m: int, restarts: int, seed: int = 0x5EED,

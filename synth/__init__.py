@@ -83,6 +83,54 @@ def gpt_tables(L: int, h: int, s: int, mbs: int, V: int):
     return f, b, a
 
 
+def gpt_memory(L: int, h: int, s: int, mbs: int, V: int):
+    """Per-sub-layer (static_bytes, stash_bytes) for the N4 memory model (DESIGN.md
+    reading R-N4), same sub-layer order as gpt_tables.
+
+    static: 16 B per parameter (bf16 weight + bf16 gradient + fp32 master weight + two
+    fp32 Adam moments); parameters: emb V*h + s*h, attn 4h^2 + 4h + 2h (LayerNorm),
+    ffn 8h^2 + 5h + 2h, head V*h + 2h (untied).
+    stash (activation checkpointing): the sub-layer's input per in-flight
+    micro-batch -- token ids (8 B each) for emb, the bf16 hidden state 2*mbs*s*h else."""
+    st: List[int] = []
+    sh: List[int] = []
+    hid = 2 * mbs * s * h
+    st.append(16 * (V * h + s * h)); sh.append(8 * mbs * s)
+    for _ in range(L):
+        st.append(16 * (4 * h * h + 6 * h)); sh.append(hid)
+        st.append(16 * (8 * h * h + 7 * h)); sh.append(hid)
+    st.append(16 * (V * h + 2 * h)); sh.append(hid)
+    return st, sh
+
+
+@dataclasses.dataclass(frozen=True)
+class DepthWorkload:
+    """NEXT N4: outer planner loop over pipeline depth with a memory model."""
+
+    name: str
+    base: Workload           # tables (its p, m are unused)
+    static_bytes: Tuple[int, ...]
+    stash_bytes: Tuple[int, ...]
+    cap_bytes: int
+    n_gpus: int
+    microbatches: int        # per iteration, over all data-parallel replicas
+
+
+def depth_config() -> DepthWorkload:
+    """GPT-2 1.3B (Table I: 24 layers, h 2048) with micro-batch size 16 on 8
+    GPUs, global batch 512 (Table IV) -> 32 micro-batches per iteration; per-GPU
+    capacity 24 GiB (the paper's RTX 3090s)."""
+    L, h, s, mbs, V = 24, 2048, 1024, 16, 50257
+    f, b, a = gpt_tables(L, h, s, mbs, V)
+    base = Workload(name="N4-gpt2-1.3b-mbs16", fwd_ns=tuple(f), bwd_ns=tuple(b),
+                    act_bytes=tuple(a), link_bytes_per_s=LINK_BYTES_PER_S, p=1, m=1,
+                    k_lo=1, k_hi=1, search="exhaustive")
+    st, sh = gpt_memory(L, h, s, mbs, V)
+    return DepthWorkload(name="N4-gpt2-1.3b-mbs16-g8-gbs512-24GiB", base=base,
+                         static_bytes=tuple(st), stash_bytes=tuple(sh), cap_bytes=24 << 30,
+                         n_gpus=8, microbatches=512 // mbs)
+
+
 def _wl(name, L, h, s, mbs, V, **kw) -> Workload:
     f, b, a = gpt_tables(L, h, s, mbs, V)
     return Workload(name=name, fwd_ns=tuple(f), bwd_ns=tuple(b), act_bytes=tuple(a),

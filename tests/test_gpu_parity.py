@@ -751,3 +751,90 @@ def test_reach_errors(ap):
                  (3, 4, 0, 2, 0, (1 << 20) + 1, 8)]:
         with pytest.raises(ap.APError):
             ap.ap_search_reachable(plan, *args, key)
+
+
+# --------------------------------------------------------------------------- N4 depth
+def test_memory_mode_random_vs_oracle(ap, oracle_mod):
+    """AP_SEARCH_MEMORY == the oracle's feasible argmin (T, rank, k), with capacities
+    from 'nothing fits' to 'everything fits', including an infeasible Alg.-1 start
+    (search_exhaustive's two-phase fallback)."""
+    from paper_conf_cluster_liulldgl22_b200.search import search_exhaustive
+    rng = np.random.default_rng(44)
+    for trial in range(14):
+        kind = ["uniform", "b3f", "small", "equal"][trial % 4]
+        n = int(rng.integers(3, 16))
+        f, b, a = synth.random_tables(700 + trial, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        st = rng.integers(0, 1 << 30, n)
+        sh = rng.integers(0, 1 << 26, n)
+        p = int(rng.integers(1, min(n, 6) + 1))
+        m = int(rng.choice([1, 2, p, p + 3, 12]))
+        k_hi = int(rng.integers(1, 4))
+        tot = int(st.sum() + min(p, m) * sh.sum())
+        for cap in (tot // 8, tot // 3, tot // 2, tot):
+            ap.ap_plan_set_memory(plan, st, sh, cap)
+            r = search_exhaustive(plan, p, m, 1, k_hi, mode=ap.AP_SEARCH_MEMORY)
+            o = M.exhaustive_mem(p, m, 1, k_hi, st, sh, cap)
+            if o["T"] is None:
+                assert r["key"] == ap.INT64_MAX, (trial, cap)
+                continue
+            assert (r["time_ns"], r["rank"], r["k"]) == (o["T"], o["rank"], o["k"]), (trial, cap)
+
+
+def test_plan_pipeline_depth_vs_oracle(ap, oracle_mod):
+    """The N4 workload (GPT-2 1.3B, mbs 16, 8 GPUs, 24 GiB): every depth's feasible
+    argmin and the chosen depth equal the oracle's (p = 8 on sampled rank windows)."""
+    import torch
+    from paper_conf_cluster_liulldgl22_b200.search import plan_pipeline_depth
+    d = synth.depth_config()
+    f, b, a = d.base.arrays()
+    plan = _plan(ap, f, b, a, d.base.link_bytes_per_s)
+    ap.ap_plan_set_memory(plan, d.static_bytes, d.stash_bytes, d.cap_bytes)
+    M = oracle_mod.Model.from_workload(d.base)
+    out = plan_pipeline_depth(plan, d.n_gpus, d.microbatches)
+    rows = {r["p"]: r for r in out["per_depth"]}
+    assert sorted(rows) == [1, 2, 4, 8]
+    for p in (1, 2, 4):
+        o = M.exhaustive_mem(p, rows[p]["m"], 1, 1, d.static_bytes, d.stash_bytes, d.cap_bytes)
+        assert rows[p]["T"] == o["T"]
+        if o["T"] is not None:
+            assert (rows[p]["rank"], rows[p]["cuts"]) == (o["rank"], [int(x) for x in o["cuts"]])
+    feas = [(rows[p]["T"], p) for p in rows if rows[p]["T"] is not None]
+    assert out["best"]["p"] == min(feas)[1]
+    # p = 8 on windows: the device feasible argmin of [lo, hi) == the oracle's
+    N = ap.ap_count(d.base.n, 8)
+    m8 = rows[8]["m"]
+    out2 = torch.empty(2, dtype=torch.int64, device="cuda")
+    # a shard keeps only candidates with T <= T_ref (the Alg.-1 partition's T when it
+    # fits; include/ap.h AP_SEARCH_MEMORY)
+    a1, _ = M.alg1(8)
+    tref = (M.T(8, m8, a1) if M.feasible(8, m8, a1, d.static_bytes, d.stash_bytes, d.cap_bytes)
+            else None)
+    r1 = oracle_mod.rank(d.base.n, 8, a1)
+    nontrivial = 0
+    for lo in (0, N // 3, N - 20000, max(0, r1 - 10000)):
+        hi = lo + 20000
+        ap.ap_search_exhaustive2(plan, 8, m8, 1, 1, lo, hi, ap.AP_SEARCH_MEMORY, out2)
+        torch.cuda.synchronize()
+        o = M.exhaustive_mem(8, m8, 1, 1, d.static_bytes, d.stash_bytes, d.cap_bytes, lo, hi)
+        if o["T"] is None or (tref is not None and o["T"] > tref):
+            assert int(out2[0]) == ap.INT64_MAX
+        else:
+            assert (int(out2[0]), int(out2[1])) == (o["T"], o["rank"])
+            nontrivial += 1
+    assert nontrivial >= 1
+
+
+def test_memory_mode_errors(ap):
+    import torch
+    f, b, a = synth.random_tables(3, 10, "uniform")
+    plan = _plan(ap, f, b, a, synth.link_for("uniform"))
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    with pytest.raises(ap.APError):  # no memory model yet
+        ap.ap_search_exhaustive_mode(plan, 3, 4, 1, 1, 0, 36, ap.AP_SEARCH_MEMORY, key)
+    with pytest.raises(ap.APError):
+        ap.ap_plan_set_memory(plan, [-1] * 10, [0] * 10, 100)
+    with pytest.raises(ap.APError):
+        ap.ap_plan_set_memory(plan, [1 << 61] * 10, [0] * 10, 100)

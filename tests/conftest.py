@@ -18,3 +18,20 @@ def oracle_mod():
     import oracle
     oracle.build()
     return oracle
+
+
+def _ensure_libap():
+    """Build libap.so in-tree if it is missing (a fresh checkout); loaded by path so the
+    package __init__ (which refuses to run without the library) is not imported."""
+    lib = os.path.join(ROOT, "paper_conf_cluster_liulldgl22_b200", "libap.so")
+    if os.path.exists(lib) or os.environ.get("AP_LIB_PATH"):
+        return
+    import importlib.util
+    spec = importlib.util.spec_from_file_location(
+        "_ap_build", os.path.join(ROOT, "paper_conf_cluster_liulldgl22_b200", "_build.py"))
+    mod = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mod)
+    mod.build()
+
+
+_ensure_libap()

@@ -51,10 +51,25 @@ def _peaks():
 
 
 def int_peak_ops(sm_mhz: float, sms: int = 148) -> float:
-    """Integer ALU roofline: 4 SMSPs x 32 lanes issue one warp
-    instruction per clock per SMSP = 128 int32 lanes/clk/SM, split between the alu
-    pipe (VIMNMX, 64/clk) and the fma pipe (VIADD/IMAD, 64/clk)."""
-    return sms * 128 * sm_mhz * 1e6
+    """Integer ALU roofline in int32 ops/s.  Per SM per clock: the alu
+    pipe retires 64 lanes (4 SMSPs x 16, rt_SMSP = 2) of instructions that each do up to
+    TWO int32 ops (VIADDMNMX = add + max, IADD3 = two adds), and the fmaheavy pipe 64
+    lanes of IMAD (one add).  Issue (1 warp-instruction/clk/SMSP = 128 lanes) is not
+    binding beyond that.  Peak = 148 x (64*2 + 64*1) = 192 int32 ops/clk/SM."""
+    return sms * 192 * sm_mhz * 1e6
+
+
+NCU_PROFILE = os.path.join(ROOT, "profiles", "ncu_sweep_c4.json")
+
+
+def _ncu_profile():
+    """Per-launch figures of the dominant kernel from the committed ncu --set full
+    capture (tools/ncu_summary.py --json writes it): DRAM bytes, issue/pipe use."""
+    try:
+        with open(NCU_PROFILE) as fh:
+            return json.load(fh)
+    except Exception:
+        return None
 
 
 def ops_per_sim(p: int, m: int, k: int) -> int:
@@ -378,9 +393,15 @@ def main():
             "frac_naive_count": (my_ops_naive / k_avg_s / peak) if k_avg_s > 0 else None,
             "kernel_ms_avg": k_avg_s * 1e3,
             "kernel_share_of_step": (kern_max / t_max) if t_max > 0 else None,
-            "peak_source": f"{sms} SMs x 128 int32 lanes/clk x sm_max {sm_max:.0f} MHz "
+            "peak_source": f"{sms} SMs x 192 int32 ops/clk (alu pipe 64 lanes x 2 ops fused "
+                           f"+ fmaheavy 64 lanes x 1 op) x sm_max {sm_max:.0f} MHz "
                            f"({peak_src} MEASURED_PEAKS.json clock)",
-            "traffic_note": "algorithmic HBM bytes per candidate = 0; see profiles/ for ncu DRAM bytes"}
+            "traffic_note": "algorithmic HBM bytes per candidate = 0; traffic = ncu "
+                            "dram__bytes_read+write of this kernel, one --set full capture"}
+    prof = _ncu_profile()
+    if prof:
+        roof["traffic"] = prof.get("dram_bytes_per_launch")
+        roof["ncu"] = prof
     out = {"metric": METRIC, "value": value, "unit": "sims/s", "n_gpus": world,
            "steps": args.steps, "warmup": args.warmup,
            "ms_per_step": 1e3 * t_max / args.steps,

@@ -377,6 +377,9 @@ typedef struct {
   int32_t rank_bits;       /* rb                                                  */
   int32_t launches;        /* kernels launched by the call                        */
   int32_t clamp_rows;      /* u32 path: steady rows between saturating clamps      */
+  int32_t clamp_first;     /* u32 path: steady rows before the first clamp (0 = clamp
+                              right after the warm-up; > m-p = no clamp at all)     */
+  int32_t clamp_final;     /* u32 path: 1 = clamp once more before the cool-down    */
 } ap_launch_info;
 void ap_last_launch(ap_launch_info* info);
 

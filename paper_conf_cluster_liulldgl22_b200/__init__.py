@@ -49,7 +49,8 @@ class ApOp(C.Structure):
 class ApLaunchInfo(C.Structure):
     _fields_ = [("fast_u32", C.c_int32), ("exact_p", C.c_int32), ("blocks", C.c_int32),
                 ("threads", C.c_int32), ("chunk", C.c_uint64), ("t_ref", C.c_int64),
-                ("rank_bits", C.c_int32), ("launches", C.c_int32), ("clamp_rows", C.c_int32)]
+                ("rank_bits", C.c_int32), ("launches", C.c_int32), ("clamp_rows", C.c_int32),
+                ("clamp_first", C.c_int32), ("clamp_final", C.c_int32)]
 
 
 def _load_lib():

@@ -631,16 +631,43 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   // R_allow = floor((2^32-1-S)/W_row) rows per clamp segment nothing wraps.  The
   // segments are: rows 0..p-1 (pieces + warm-up + first 1F1B row), blocks of
   // clamp_rows steady rows, and the p-1 cool-down rows.
+  //
+  // Schedule (clamp_first / clamp_rows / clamp_final): A0 = rows a value may grow from 0 (the
+  // first segment: p warm-up rows + clamp_first steady rows), r_allow = rows from S
+  // (every later segment; the last one plus the p cool-down rows).  With C4 the whole
+  // schedule is ONE clamp.
   const uint64_t S = (uint64_t)tref + 1;
   const unsigned __int128 wrow = (unsigned __int128)(plan->sum_f + plan->sum_b) +
                                  (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
   const unsigned __int128 lim = ((unsigned __int128)1 << 32) - 1;
-  const uint64_t r_allow = (S >= lim) ? 0 : (uint64_t)((lim - S) / wrow);
-  int want_u32 = r_allow >= (uint64_t)p && r_allow >= 1;
-  int clamp_rows = (int)(r_allow < (uint64_t)m ? r_allow : (uint64_t)m);
-  if (clamp_rows >= 8) clamp_rows &= ~7;  // whole unrolled blocks
-  else if (clamp_rows >= 4) clamp_rows &= ~3;
-  if (clamp_rows < 1) clamp_rows = 1;
+  const int64_t a0 = (int64_t)(lim / wrow);
+  const int64_t r_allow = (S >= lim) ? -1 : (int64_t)((lim - S) / wrow);
+  int want_u32 = r_allow >= (int64_t)p && r_allow >= 1;
+  int clamp_first = 0, clamp_rows = 1, clamp_final = 1;
+  if (want_u32) {
+    auto whole = [](int64_t r) { return r >= 8 ? (r & ~int64_t(7)) : (r >= 4 ? (r & ~int64_t(3)) : r); };
+    const int64_t steady = m - p;
+    if (steady + 2 * (int64_t)p <= a0) {
+      clamp_first = (int)steady + 1;  // no clamp at all
+      clamp_rows = m;
+      clamp_final = 0;
+    } else {
+      int64_t s1 = a0 - p;
+      if (s1 >= 1) s1 = whole(s1 < steady ? s1 : steady);
+      else s1 = 0;  // clamp right after the warm-up
+      clamp_first = (int)s1;
+      const int64_t L = steady - s1;
+      int64_t every = L < r_allow ? L : r_allow;
+      every = every >= 1 ? whole(every) : 1;
+      clamp_rows = (int)every;
+      if (L == 0) {
+        clamp_final = 1;
+      } else {
+        const int64_t last = L - every * ((L - 1) / every);
+        clamp_final = (last + p > r_allow) ? 1 : 0;
+      }
+    }
+  }
   // test/bench overrides: AP_SWEEP=int64 disables the u32 path, AP_SWEEP=generic
   // also the p-specialised kernel (both remain exact)
   const char* ov = getenv("AP_SWEEP");
@@ -654,6 +681,11 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   } else {
     AP_CUDA(sc.get((void**)&rec, 16 * (size_t)apk::sweep_max_blocks(plan->device)));
   }
+  // warp-dynamic work cursor for the p-specialised sweep;
+  // AP_SWEEP_SCHED=static keeps the one-chunk-per-thread split (A/B measurements)
+  unsigned long long* ctr = nullptr;
+  const char* sched = getenv("AP_SWEEP_SCHED");
+  if (!(sched && strcmp(sched, "static") == 0)) AP_CUDA(sc.get((void**)&ctr, 16));
   AP_CUDA(g_timer.record(0, s, plan->device));
   if (mem) {
     want_u32 = 0;  // memory mode: the generic exact kernel with the feasibility filter
@@ -662,7 +694,8 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, S, rb, want_u32,
                             clamp_rows, force_generic, mem ? AP_SEARCH_FULL : mode,
                             reinterpret_cast<unsigned long long*>(key), s, &sp, rec,
-                            mem ? plan->d_mem : nullptr, plan->mem_cap));
+                            mem ? plan->d_mem : nullptr, plan->mem_cap, ctr, clamp_first,
+                            clamp_final));
   if (rec) {
     AP_CUDA(apk::launch_reduce2(rec, sp.blocks, reinterpret_cast<long long*>(out2), s));
     ++launches;
@@ -679,6 +712,8 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   info.t_ref = tref;
   info.rank_bits = rb;
   info.clamp_rows = sp.fast_u32 ? clamp_rows : 0;
+  info.clamp_first = sp.fast_u32 ? clamp_first : 0;
+  info.clamp_final = sp.fast_u32 ? clamp_final : 0;
   info.launches = launches;
   g_last = info;
   return AP_OK;

@@ -15,6 +15,7 @@
 // Every kernel starts with the K4 prologue (TMA bulk copy of the tables into
 // shared memory + warp-shuffle prefix sums), see ap_device.cuh.
 #include <climits>
+#include <cstdlib>
 #include <cstdio>
 
 #include "ap_device.cuh"
@@ -144,6 +145,14 @@ AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const 
   }
 }
 
+// Saturating-clamp schedule of the u32 sweep, computed by the host:
+// `first` steady rows before the first clamp (0 = clamp right after the warm-up), then
+// a clamp every `every` steady rows, and `fin` = clamp once more at the end of the
+// steady rows.  Ignored for 64-bit V.
+struct ClampSched {
+  int first, every, fin;
+};
+
 // Everything after the pieces, for p == P, m >= P: warm-up rows, the first 1F1B row,
 // the fused steady steps and the fused cool-down.
 //  REV = false: input FF = finishes of F(x, 0, k-1); returns T = end of B(0, m-1).
@@ -156,8 +165,8 @@ AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const 
 //               F(x,1)),   G[P-1] = F'(P-1, m-1) (via B(P-1,0)),
 //      so that T(k) = max_x (FF_x(k) + G[x]) for every k.
 template <int P, typename V, bool REV>
-AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V S, int CR,
-                           uint32_t one, V (&G)[P]) {
+AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V S,
+                           ClampSched cs, uint32_t one, V (&G)[P]) {
   using O = XOps<V>;
   V L[P];
   // warm-up rows r = 1..P-2: stage x <= r-1 does F(x, r-x); L == FF here
@@ -173,24 +182,27 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
 #pragma unroll
   for (int x = P - 2; x >= 1; --x) FF[x] = O::ad(O::mx(FF[x - 1], L[x]), wF[x], one);
   if (P >= 2) FF[0] = O::ad(L[0], wF[0], one);
-  clamp_ff<P, V>(FF, S);
   // fused steps r = P-1..m-2: backward pass of row r + forward pass of row r+1,
-  // clamped (u32) every CR steps: the host's no-wrap bound S + CR * W_row < 2^32
-  //
+  // u32: clamped on the host's schedule `cs` (no-wrap bounds)
   {
     constexpr int U = (P <= 8) ? 8 : 4;
     const V wBF0 = wB[0] + wF[0];
     int rem = m - P;
+    if (sizeof(V) == 4 && cs.first == 0) clamp_ff<P, V>(FF, S);
+    int seg = (sizeof(V) == 4 && cs.first > 0) ? cs.first : cs.every;
+    if (sizeof(V) != 4) seg = rem;
     while (rem > 0) {
-      int blk = rem < CR ? rem : CR;
+      int blk = rem < seg ? rem : seg;
       rem -= blk;
       for (; blk >= U; blk -= U) {
 #pragma unroll
         for (int u = 0; u < U; ++u) mstep<P, V>(FF, wF, wB, wBF0, one);
       }
       for (; blk > 0; --blk) mstep<P, V>(FF, wF, wB, wBF0, one);
-      clamp_ff<P, V>(FF, S);
+      if (rem > 0 || cs.fin) clamp_ff<P, V>(FF, S);
+      seg = cs.every;
     }
+    if (m == P && cs.fin && cs.first != 0) clamp_ff<P, V>(FF, S);
   }
   // cool-down, fused the same way: step t = 0..P-1 is the backward pass of row
   // r = m-1+t plus the forward pass of row r+1, which only stages x >= t+1 still
@@ -240,10 +252,11 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
 // Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
 template <int P, typename V>
 AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const int (&c)[P + 1],
-                         const V* sPf, const V* sC, uint32_t Mk, V S, int CR, uint32_t one) {
+                         const V* sPf, const V* sC, uint32_t Mk, V S, ClampSched cs,
+                         uint32_t one) {
   V FF[P], G[P];
   pieces<P, V>(k, wF, c, sPf, sC, Mk, one, FF);
-  return sweep_tail<P, V, false>(m, FF, wF, wB, S, CR, one, G);
+  return sweep_tail<P, V, false>(m, FF, wF, wB, S, cs, one, G);
 }
 
 struct SweepArgs {
@@ -253,12 +266,15 @@ struct SweepArgs {
   uint64_t S;
   int rb;
   unsigned long long* key;
-  int clamp_rows;  // u32 path: rows between saturating clamps (>= 1)
+  int clamp_rows;  // u32 path: steady rows between saturating clamps (>= 1)
+  int clamp_first; // u32 path: steady rows before the first clamp (0: right after warm-up)
+  int clamp_final; // u32 path: clamp at the end of the steady rows
   uint32_t one;    // = 1 (adds are plain operators; kept for the XOps interface)
   int mode;        // 0 full, 1 k-factored, 2 k-factored + lower-bound skipping
   unsigned long long* rec;  // two-phase: per-CTA (T, index) records instead of `key`
   const int64_t* mem;       // memory filter (generic kernel): [2][n+1] prefix sums
   int64_t mem_cap;
+  unsigned long long* ctr;  // non-null: warp-dynamic work cursor (zeroed), chunk = ranks/lane/unit
 };
 
 AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
@@ -377,6 +393,11 @@ __global__ void k_key2_select(const long long* local, const long long* t_star, l
 }
 
 template <int P, typename V>
+__device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1,
+                                            const V* sPf, const V* sPb, const V* sC,
+                                            const uint32_t* s_mk, V& bestT, uint64_t& bestIdx);
+
+template <int P, typename V>
 #ifndef AP_SWEEP_MINB
 #define AP_SWEEP_MINB (P <= 8 ? 3 : 2)
 #endif
@@ -399,15 +420,44 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
     s_mk[threadIdx.x] = (threadIdx.x <= 1) ? 0xffffffffu : (uint32_t)((1ull << 32) / threadIdx.x);
   __syncthreads();
 
-  const int m = A.m, k_lo = A.k_lo, k_hi = A.k_hi;
-  const uint64_t K = (uint64_t)(k_hi - k_lo + 1);
   const V S = (V)A.S;
   V bestT = S;
   uint64_t bestIdx = 0;
-  const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const uint64_t r0 = A.rank_lo + tid * A.chunk;
-  if (r0 < A.rank_hi) {
-    const uint64_t r1 = min(r0 + A.chunk, A.rank_hi);
+  if (A.ctr) {
+    // persistent, warp-dynamic: a warp claims unit u = 32 lanes x `chunk` consecutive
+    // ranks from the global cursor, so warps the scheduler favoured do not leave the
+    // SM under-occupied at the end
+    const int lane = threadIdx.x & 31;
+    for (;;) {
+      unsigned long long u = 0;
+      if (lane == 0) u = atomicAdd(A.ctr, 1ull);
+      u = __shfl_sync(0xffffffffu, u, 0);
+      const uint64_t span = A.rank_hi - A.rank_lo;
+      if (u * 32ull >= (span + A.chunk - 1) / A.chunk) break;
+      const uint64_t r0 = A.rank_lo + (u * 32ull + (uint64_t)lane) * A.chunk;
+      if (r0 < A.rank_hi)
+        sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), sPf, sPb, sC, s_mk, bestT, bestIdx);
+    }
+  } else {
+    const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const uint64_t r0 = A.rank_lo + tid * A.chunk;
+    if (r0 < A.rank_hi)
+      sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), sPf, sPb, sC, s_mk, bestT, bestIdx);
+  }
+  sweep_result(A, bestT < S, (uint64_t)bestT, bestIdx);
+}
+
+// Ranks [r0, r1) x k of one thread: unrank r0, then lex successors (a2-a7).
+template <int P, typename V>
+__device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1,
+                                            const V* sPf, const V* sPb, const V* sC,
+                                            const uint32_t* s_mk, V& bestT, uint64_t& bestIdx) {
+  const int n = A.t.n;
+  const int m = A.m, k_lo = A.k_lo, k_hi = A.k_hi;
+  const uint64_t K = (uint64_t)(k_hi - k_lo + 1);
+  const V S = (V)A.S;
+  const ClampSched cs{A.clamp_first, A.clamp_rows, A.clamp_final};
+  {
     // unrank r0 (reading O7 lex order)
     int c[P + 1];
     c[0] = 0;
@@ -467,7 +517,7 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
       if (live && A.mode == 0) {
         for (int k = k_lo; k <= k_hi; ++k) {
           const uint32_t Mk = s_mk[k];
-          const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, S, A.clamp_rows, A.one);
+          const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, S, cs, A.one);
           if (Tc < bestT) {
             bestT = Tc;
             bestIdx = base + (uint64_t)(k - k_lo);
@@ -486,7 +536,7 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
           FF0[0] = rF[0];
 #pragma unroll
           for (int x = 1; x < P; ++x) FF0[x] = FF0[x - 1] + rF[x];
-          sweep_tail<P, V, true>(m, FF0, rF, rB, S, A.clamp_rows, A.one, G);
+          sweep_tail<P, V, true>(m, FF0, rF, rB, S, cs, A.one, G);
         }
         for (int k = k_lo; k <= k_hi; ++k) {
           V Tc;
@@ -500,7 +550,7 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
               Tc = v > Tc ? v : Tc;
             }
           } else {
-            Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, s_mk[k], S, A.clamp_rows, A.one);
+            Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, s_mk[k], S, cs, A.one);
           }
           if (Tc < bestT) {
             bestT = Tc;
@@ -520,7 +570,6 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
       }
     }
   }
-  sweep_result(A, bestT < S, (uint64_t)bestT, bestIdx);
 }
 
 // Generic exhaustive sweep: runtime p <= P, any m, exact int64.
@@ -1741,10 +1790,32 @@ static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int
   occ = occ < 1 ? 1 : occ;
   const uint64_t nr = A.rank_hi - A.rank_lo;
   const uint64_t target = (uint64_t)num_sms(dev) * occ * threads;
-  A.chunk = (nr + target - 1) / target;
-  if (A.chunk == 0) A.chunk = 1;
-  const uint64_t nthreads = (nr + A.chunk - 1) / A.chunk;
-  const uint64_t blocks = (nthreads + threads - 1) / threads;
+  uint64_t blocks;
+  if (A.ctr) {
+    // persistent warp-dynamic grid (one wave): units of 32 lanes x chunk ranks, about
+    // kUnitsPerWarp units per warp so the end-of-kernel imbalance is ~1/kUnitsPerWarp
+    // of a warp's work, while the per-unit unrank stays negligible
+    uint64_t kUnitsPerWarp = 128, kMinSims = 128;
+    if (const char* e = getenv("AP_SWEEP_UPW")) kUnitsPerWarp = strtoull(e, nullptr, 10);
+    if (const char* e = getenv("AP_SWEEP_MINSIMS")) kMinSims = strtoull(e, nullptr, 10);
+    const uint64_t K = (uint64_t)(A.k_hi - A.k_lo + 1);
+    A.chunk = (nr + target * kUnitsPerWarp - 1) / (target * kUnitsPerWarp);
+    const uint64_t cmin = (kMinSims + K - 1) / K;  // amortise the per-unit unrank
+    if (A.chunk < cmin) A.chunk = cmin;
+    if (A.chunk == 0) A.chunk = 1;
+    const uint64_t units = (nr + 32 * A.chunk - 1) / (32 * A.chunk);
+    const uint64_t need = (units * 32 + threads - 1) / threads;
+    blocks = (uint64_t)num_sms(dev) * occ;
+    if (blocks > need) blocks = need;
+    if (blocks < 1) blocks = 1;
+    cudaError_t em = cudaMemsetAsync(A.ctr, 0, sizeof(unsigned long long), s);
+    if (em != cudaSuccess) return em;
+  } else {
+    A.chunk = (nr + target - 1) / target;
+    if (A.chunk == 0) A.chunk = 1;
+    const uint64_t nthreads = (nr + A.chunk - 1) / A.chunk;
+    blocks = (nthreads + threads - 1) / threads;
+  }
   if (A.rec && blocks > (uint64_t)sweep_max_blocks(dev)) return cudaErrorInvalidValue;
   k_sweep_exact<P, V><<<(unsigned)blocks, threads, smem, s>>>(A);
   sp->blocks = (int)blocks;
@@ -1824,11 +1895,13 @@ cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, u
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
                          SweepPlan* sp, unsigned long long* rec, const int64_t* mem,
-                         int64_t mem_cap) {
+                         int64_t mem_cap, unsigned long long* ctr, int clamp_first,
+                         int clamp_final) {
   int dev = 0;
   cudaGetDevice(&dev);
-  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key, clamp_rows < 1 ? 1 : clamp_rows, 1u, mode, rec,
-              mem, mem_cap};
+  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key,
+              clamp_rows < 1 ? 1 : clamp_rows, clamp_first < 0 ? 0 : clamp_first,
+              clamp_first < 0 ? 1 : clamp_final, 1u, mode, rec, mem, mem_cap, ctr};
   const bool exact = !mem && has_exact(p) && m >= p && (!force_generic || mode != 0);
   sp->exact_p = exact ? 1 : 0;
   sp->fast_u32 = (exact && want_u32) ? 1 : 0;

@@ -40,11 +40,18 @@ struct SweepPlan {
 };
 // Exhaustive sweep of ranks [rank_lo, rank_hi) x k in [k_lo, k_hi].  S = T_ref + 1:
 // a candidate with T >= S can never win.  atomicMin into *key (init it first).
+// ctr (8 B, device): the p-specialised kernel then runs persistent with warp-dynamic
+// work units (zeroed here, stream-ordered); null = static per-thread chunks.
+// u32 clamp schedule: clamp_first steady rows before the first clamp (-1: legacy =
+// clamp after the warm-up and at the end), then every clamp_rows, clamp_final = one
+// more clamp at the end of the steady rows.
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
                          uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
                          SweepPlan* plan_out, unsigned long long* rec = nullptr,
-                         const int64_t* mem = nullptr, int64_t mem_cap = 0);
+                         const int64_t* mem = nullptr, int64_t mem_cap = 0,
+                         unsigned long long* ctr = nullptr, int clamp_first = -1,
+                         int clamp_final = 1);
 
 // Two-phase reduction (NEXT N3).  With `rec` (u64[2 * sweep_max_blocks(dev)]) passed
 // to launch_sweep, each CTA stores its lexicographic min (T, index) there instead of

@@ -357,9 +357,54 @@ def test_exhaustive_u32_tight_bound_saturates(ap, oracle_mod, monkeypatch):
         o = M.exhaustive(p, m, 1, k_hi)
         res = ap.ap_decode(plan, 0, p, m, 1, k_hi, key=key)
         assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
-        if info["fast_u32"] and info["clamp_rows"] < m - p:
+        # a schedule with more than one clamp inside the steady rows
+        if info["fast_u32"] and info["clamp_first"] + info["clamp_rows"] < m - p:
             hits += 1
     assert hits >= 3
+
+
+def test_exhaustive_u32_clamp_schedules(ap, oracle_mod, monkeypatch):
+    """The host's saturating-clamp schedule (no clamp / one clamp /
+    clamp right after the warm-up / a final clamp before the cool-down): over cost
+    scales that produce every schedule, the u32
+    key equals the int64 sweep's and the oracle's argmin, in all three search modes."""
+    rng = np.random.default_rng(77)
+    seen = set()
+    for trial in range(40):
+        n = int(rng.integers(9, 13))
+        p = int(rng.choice([3, 4, 5, 8]))
+        p = min(p, n - 1)
+        m = int(rng.integers(p, p + 40))
+        scale = float(2.0 ** rng.uniform(10, 26))
+        f = (rng.uniform(0.3, 1.0, n) * scale).astype(np.int64)
+        b = (rng.uniform(0.3, 1.0, n) * 3 * scale).astype(np.int64)
+        a = rng.integers(0, 1 << 22, n).astype(np.int64)
+        plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+        k_hi = int(rng.integers(1, 4))
+        monkeypatch.delenv("AP_SWEEP", raising=False)
+        key = _search(ap, plan, p, m, 1, k_hi)
+        info = ap.ap_last_launch()
+        keys = [_search_mode(ap, plan, p, m, 1, k_hi, md) for md in (1, 2)]
+        monkeypatch.setenv("AP_SWEEP", "int64")
+        key64 = _search(ap, plan, p, m, 1, k_hi)
+        assert key == key64 == keys[0] == keys[1], (trial, info)
+        if info["fast_u32"]:
+            steady = m - p
+            if info["clamp_first"] > steady:
+                kind = "none"
+            elif info["clamp_first"] == 0:
+                kind = "after-warmup"
+            else:
+                kind = "first-segment"
+            seen.add(kind)
+            if info["clamp_final"]:
+                seen.add("final")
+            if trial % 4 == 0:
+                M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+                o = M.exhaustive(p, m, 1, k_hi)
+                res = ap.ap_decode(plan, 0, p, m, 1, k_hi, key=key)
+                assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+    assert {"none", "first-segment", "final"} <= seen, seen
 
 
 def test_key_layout_matches_python_helpers(ap):

@@ -930,18 +930,20 @@ AP_DEV_INLINE uint32_t sim_fast_bits(int m, const uint32_t (&wF)[P], const uint3
     int blk = rem < CR ? rem : CR;
     rem -= blk;
     for (; blk > 0; --blk) {
-      uint32_t wordB = 0, wordF = 0, nF[P];
+      // one compare per stage: the F bit x+1 is gt_x, the B bit 16+x its complement,
+      // formed once per row from wordF
+      uint32_t wordF = 0, nF[P];
       uint32_t b = FF[P - 1] + wB[P - 1];
 #pragma unroll
       for (int x = P - 2; x >= 0; --x) {
         const bool gt = FF[x] > b;
-        wordF |= (gt ? 1u : 0u) << (x + 1);
-        wordB |= (gt ? 0u : 1u) << (x + 16);
-        const uint32_t M = gt ? FF[x] : b;
+        if (gt) wordF |= 1u << (x + 1);
+        const uint32_t M = max(FF[x], b);
         nF[x + 1] = M + wF[x + 1];
         b = M + wB[x];
       }
       nF[0] = b + wF[0];
+      const uint32_t wordB = ((~wordF >> 1) & ((1u << (P - 1)) - 1u)) << 16;
       br.base[(size_t)r * br.stride] = nxt | wordB;
       nxt = wordF;
       ++r;
@@ -980,6 +982,71 @@ AP_DEV_INLINE uint32_t sim_fast_bits(int m, const uint32_t (&wF)[P], const uint3
     ++r;
   }
   return b;
+}
+
+// backtrack_master (ap_device.cuh) specialised to the fast path: p == P, k == 1,
+// m >= P (so w_x = P-1-x, W0 = P-1), m <= 32767.  The same walk and the same reading
+// (O5 tie rule, O6 master = most 1F1B-phase path ops, ties -> higher stage, none ->
+// P-1), but the per-stage counts live in registers: the path stays on one stage for
+// a run of ops, so a run counter is flushed into 16-bit fields of NW words only when
+// the path changes stage (unrolled select, no local memory).
+template <int P>
+AP_DEV_INLINE int backtrack_master_fast(int m, BitsRef br) {
+  constexpr int NW = (P + 1) / 2;
+  uint32_t cw[NW];
+#pragma unroll
+  for (int w = 0; w < NW; ++w) cw[w] = 0;
+  auto flush = [&](int x, uint32_t run) {
+    const uint32_t inc = run << (16 * (x & 1));
+#pragma unroll
+    for (int w = 0; w < NW; ++w) cw[w] += (w == (x >> 1)) ? inc : 0u;
+  };
+  int kind = 1, x = 0, j = m - 1;
+  uint32_t run = 0;
+  for (;;) {
+    const int wx = P - 1 - x;
+    const int row = kind ? (j + P - 1) : (j + x);
+    const uint32_t word = br.base[(size_t)row * br.stride];
+    run += kind ? (j < m - wx ? 1u : 0u) : (j >= wx ? 1u : 0u);
+    if (kind == 0 && j == 0 && x == 0) break;  // the source F(0, 0)
+    const bool cross = kind ? (x < P - 1 && ((word >> (x + 16)) & 1u))
+                            : (x > 0 && (j == 0 || ((word >> x) & 1u)));
+    if (cross) {
+      flush(x, run);
+      run = 0;
+      x += kind ? 1 : -1;
+      continue;
+    }
+    if (kind) {
+      const int jf = j + wx;
+      if (jf <= m - 1) {  // F(x, y + w_x) just before it in the same row
+        kind = 0;
+        j = jf;
+      } else if (j >= 1) {  // previous BP of the stage
+        j = j - 1;
+      } else {  // w_x = m cannot happen here (m >= P > w_x); kept for symmetry
+        kind = 0;
+        j = m - 1;
+      }
+    } else if (j > wx) {  // 1F1B: the previous op is B(x, j - w_x - 1)
+      kind = 1;
+      j = j - wx - 1;
+    } else {  // warm-up: F(x, j-1)
+      j = j - 1;
+    }
+  }
+  flush(x, run);
+  int best = P - 1;
+  uint32_t bc = (cw[(P - 1) >> 1] >> (16 * ((P - 1) & 1))) & 0xffffu;
+#pragma unroll
+  for (int xx = P - 2; xx >= 0; --xx) {
+    const uint32_t c = (cw[xx >> 1] >> (16 * (xx & 1))) & 0xffffu;
+    if (c > bc) {
+      best = xx;
+      bc = c;
+    }
+  }
+  return best;
 }
 
 struct HeurArgs {
@@ -1180,8 +1247,13 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
     } else {
       Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
     }
-    int len;
-    const int Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+    int Mc;
+    if constexpr (FAST) {
+      Mc = backtrack_master_fast<P>(m, br);
+    } else {
+      int len;
+      Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+    }
     ++rsims;
     bool ready;  // true: the next candidate is in cand; false: the restart is finished
     if (phase == 1) {
@@ -1948,7 +2020,8 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
   cudaGetDevice(&dev);
   // counter[0]: restart cursor of the first pass; counter[1]: cursor of the redo
   // pass; counter[2]: redo count; counter[3..]: redo ids (caller zeroes [0..2])
-  const bool fast = fastS > 0 && pick_P(p) == p && p >= 2 && p <= 16 && m >= p && !replay_cuts;
+  const bool fast = fastS > 0 && pick_P(p) == p && p >= 2 && p <= 16 && m >= p && m <= 32767 &&
+                    !replay_cuts;
   HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts, sims,
              best_out, fastS, fastCR < 1 ? 1 : fastCR, nullptr, adjust_mode};
   const uint64_t R = r_hi - r_lo;

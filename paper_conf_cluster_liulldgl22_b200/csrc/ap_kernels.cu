@@ -1328,6 +1328,246 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
 }
 
 // ===========================================================================
+// K3p heuristic restarts as a per-CTA simulation pool (adjust_mode 0, u32 fast path,
+// p == P, m >= P).  In k_heur one lane owns one restart, so a warp
+// runs as long as its longest walk and its lanes simulate out of step.  Here a CTA
+// owns NS restart slots.  One thread per slot advances its walk (reading O9, in
+// exactly k_heur's order) and emits simulation jobs -- the start, or the up to four
+// children a, a', b, b' of a step -- into a shared-memory ring.  Every pass each of
+// the NT threads simulates one queued job, all in step.  A slot whose jobs are all
+// done advances at the next pass; free slots refill from the global restart cursor.
+namespace hpool {
+constexpr int NT = 256;   // threads per CTA = jobs simulated per pass
+constexpr int NS = 96;    // restart slots per CTA
+constexpr int RING = 512; // job ring, >= 4 * NS
+}  // namespace hpool
+
+// Child idx (0 a, 1 a', 2 b, 3 b') of `cur` with master i (
+// reading Q17), as k_heur's gen_child; false if invalid or a duplicate.
+// reading Q17), as k_heur's gen_child, built in place in shared memory (no local
+// arrays); false if invalid or a duplicate.
+AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
+                              const int16_t* s_arg, int16_t* cand) {
+  if (cur[i + 1] - cur[i] < 2) return false;
+  for (int x = 0; x <= p; ++x) cand[x] = cur[x];
+  int j, e;
+  if (idx <= 1) {
+    cand[i] += 1;  // first block of stage i -> stage i-1
+    if (idx == 0) return true;
+    if (i - 1 < 1) return false;
+    j = i - 1;  // Alg. 1 on [0, c_{i-1}) with i-1 stages
+  } else {
+    if (i > p - 2) return false;
+    cand[i + 1] -= 1;  // last block of stage i -> stage i+1
+    if (idx == 2) return true;
+    j = i;  // Alg. 1 on [0, c_i) with i stages
+  }
+  e = cand[j];
+  bool diff = false;
+  for (int jj = j; jj >= 2; --jj) {  // Algorithm 1 line 15 (alg1_prefix)
+    const int st = s_arg[e * P1 + jj];
+    cand[jj - 1] = (int16_t)st;
+    diff = diff || (st != cur[jj - 1]);
+    e = st;
+  }
+  return diff;
+}
+
+template <int P>
+__global__ void __launch_bounds__(hpool::NT, 2) k_heur_pool(HeurArgs A) {
+  using namespace hpool;
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int n = A.t.n, p = P, m = A.m, P1 = P + 1;
+  int16_t* s_arg = reinterpret_cast<int16_t*>(smem + ((used + 15) & ~size_t(15)));
+  const int narg = (n + 1) * P1;
+  int32_t* s_a1 = reinterpret_cast<int32_t*>(s_arg + ((narg + 7) & ~7));
+  uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_a1 + 32);
+  // slot state: cut vectors [slot][0 cur | 1 best | 2+idx child idx][P+1]
+  __shared__ int16_t s_cuts[NS][6][P + 1];
+  __shared__ uint32_t s_chT[NS][4];
+  __shared__ int8_t s_chM[NS][4];
+  __shared__ uint32_t s_r[NS], s_bestT[NS];
+  __shared__ int s_pend[NS];
+  __shared__ int8_t s_state[NS], s_curM[NS], s_valid[NS], s_aband[NS];
+  __shared__ int s_steps[NS], s_nsims[NS];
+  __shared__ uint16_t s_ring[RING];
+  __shared__ int s_head, s_tail, s_stop;
+  const int tid = threadIdx.x;
+  for (int e = tid; e < narg; e += NT) s_arg[e] = A.arg[e];
+  for (int e = tid; e < p - 1; e += NT) s_a1[e] = A.alg1[e];
+  for (int s = tid; s < NS; s += NT) s_state[s] = 0;
+  if (tid == 0) {
+    s_head = 0;
+    s_tail = 0;
+    s_stop = 0;
+  }
+  __syncthreads();
+  const BitsRef br{s_bits + tid, NT};
+  const int smax = n * p;
+  unsigned long long my_key = 0x7fffffffffffffffull;
+  unsigned int my_sims = 0;
+
+  for (;;) {
+    // ---- phase A: advance the walks whose jobs are all done, refill free slots
+    if (tid < NS) {
+      const int s = tid;
+      int st = s_state[s];
+      if (st != 0 && s_pend[s] == 0) {
+        if (s_aband[s]) {
+          // a simulation saturated: the exact int64 pass redoes the whole restart
+          const unsigned int slot = atomicAdd(&A.redo[0], 1u);
+          A.redo[1 + slot] = s_r[s];
+          st = 0;
+        } else {
+          int16_t* cur = s_cuts[s][0];
+          int curM, steps, nsims;
+          uint32_t bestT;
+          bool walk = true;
+          if (st == 1) {  // the start was simulated
+            curM = s_chM[s][0];
+            bestT = s_chT[s][0];
+            for (int x = 0; x <= P; ++x) {
+              cur[x] = s_cuts[s][2][x];
+              s_cuts[s][1][x] = cur[x];
+            }
+            steps = 0;
+            nsims = 1;
+          } else {  // the children of a step were simulated: visit them in child order
+            curM = s_curM[s];
+            bestT = s_bestT[s];
+            steps = s_steps[s];
+            nsims = s_nsims[s];
+            const int valid = s_valid[s];
+            uint32_t selT = 0xffffffffu;
+            int sel = -1, selM = 0;
+            for (int idx = 0; idx < 4; ++idx) {
+              if (!((valid >> idx) & 1)) continue;
+              ++nsims;
+              const uint32_t Tc = s_chT[s][idx];
+              const int Mc = s_chM[s][idx];
+              if (Tc < bestT) {
+                bestT = Tc;
+                for (int x = 0; x <= P; ++x) s_cuts[s][1][x] = s_cuts[s][2 + idx][x];
+              }
+              if (Mc <= curM && Tc < selT) {
+                selT = Tc;
+                selM = Mc;
+                sel = idx;
+              }
+            }
+            if (sel < 0) {
+              walk = false;  // no child qualifies
+            } else {
+              for (int x = 0; x <= P; ++x) cur[x] = s_cuts[s][2 + sel][x];
+              curM = selM;
+            }
+          }
+          // next step (k_heur's begin_step with adjust_mode 0): the step cap, stop at
+          // master 0, else the children of step 3
+          int valid = 0, nj = 0;
+          if (walk && steps < smax && curM != 0) {
+            ++steps;
+            for (int idx = 0; idx < 4; ++idx)
+              if (pool_child(cur, idx, curM, p, P1, s_arg, s_cuts[s][2 + idx])) {
+                valid |= 1 << idx;
+                ++nj;
+              }
+          }
+          if (nj > 0) {
+            const int at = atomicAdd(&s_tail, nj);
+            int q = 0;
+            for (int idx = 0; idx < 4; ++idx)
+              if ((valid >> idx) & 1) s_ring[(at + q++) & (RING - 1)] = (uint16_t)(s * 4 + idx);
+            s_pend[s] = nj;
+            s_valid[s] = (int8_t)valid;
+            s_curM[s] = (int8_t)curM;
+            s_bestT[s] = bestT;
+            s_steps[s] = steps;
+            s_nsims[s] = nsims;
+            st = 2;
+          } else {  // the restart is finished
+            const uint32_t r = s_r[s];
+            my_sims += (unsigned int)nsims;
+            my_key = min(my_key, ((unsigned long long)bestT << 20) | r);
+            if (A.best_out)
+              for (int x = 1; x <= p - 1; ++x)
+                A.best_out[(size_t)(r - A.r_lo) * (p - 1) + (x - 1)] = s_cuts[s][1][x];
+            st = 0;
+          }
+        }
+      }
+      if (st == 0 && !s_stop) {
+        const uint32_t r = atomicAdd(A.counter, 1u) + A.r_lo;
+        if (r >= A.r_hi) {
+          s_stop = 1;
+        } else {
+          // restart start: Alg. 1 (r = 0) or the seeded perturbation (reading Q21)
+          int prev = 0;
+          s_cuts[s][2][0] = 0;
+          s_cuts[s][2][P] = (int16_t)n;
+          for (int x = 1; x <= p - 1; ++x) {
+            int64_t v = s_a1[x - 1];
+            if (r != 0) {
+              const uint64_t u = splitmix64(A.seed ^ ((uint64_t)r << 32) ^ (uint64_t)x);
+              v += (int64_t)(u % (uint64_t)(2 * A.radius + 1)) - A.radius;
+              v = v < prev + 1 ? prev + 1 : v;
+              v = v > n - (p - x) ? n - (p - x) : v;
+            }
+            s_cuts[s][2][x] = (int16_t)v;
+            prev = (int)v;
+          }
+          s_r[s] = r;
+          s_aband[s] = 0;
+          s_pend[s] = 1;
+          const int at = atomicAdd(&s_tail, 1);
+          s_ring[at & (RING - 1)] = (uint16_t)(s * 4);
+          st = 1;
+        }
+      }
+      s_state[s] = (int8_t)st;
+    }
+    if (!__syncthreads_or(tid < NS && s_state[tid] != 0)) break;
+    // ---- phase B: one queued job per thread, all simulated in step
+    const int head = s_head;
+    const int nj = min(s_tail - head, NT);
+    if (tid < nj) {
+      const int job = s_ring[(head + tid) & (RING - 1)];
+      const int s = job >> 2, idx = job & 3;
+      int cc[P + 1];
+#pragma unroll
+      for (int x = 0; x <= P; ++x) cc[x] = s_cuts[s][2 + idx][x];
+      int64_t F[P], B[P], C[P];
+      stage_costs<P>(T, p, cc, F, B, C);
+      uint32_t wF[P], wB[P];
+#pragma unroll
+      for (int x = 0; x < P; ++x) {
+        wF[x] = (uint32_t)(F[x] + ((x > 0) ? C[x - 1] : 0));
+        wB[x] = (uint32_t)(B[x] + C[x]);
+      }
+      const uint32_t t32 = sim_fast_bits<P>(m, wF, wB, A.S, A.CR, br);
+      if (t32 >= A.S) {
+        s_aband[s] = 1;
+      } else {
+        s_chT[s][idx] = t32;
+        s_chM[s][idx] = (int8_t)backtrack_master_fast<P>(m, br);
+      }
+      atomicSub(&s_pend[s], 1);
+    }
+    __syncthreads();
+    if (tid == 0) s_head = head + nj;
+  }
+  if (A.sims) {
+    unsigned long long sm = my_sims;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) sm += __shfl_xor_sync(0xffffffffu, sm, o);
+    if ((tid & 31) == 0 && sm) atomicAdd(A.sims, sm);
+  }
+  block_min_atomic(my_key, A.key);
+}
+
+// ===========================================================================
 // K3r reachable-set search (NEXT N1; reading R-N1): the literal reading of
 // PAPER.md:196, every qualifying child is processed.  One QUAD (4 lanes) per restart,
 // breadth-first: the quad pops the next queued scheme with master i > 0, lane q
@@ -2010,6 +2250,28 @@ static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev, uint64_t n
   return cudaGetLastError();
 }
 
+template <int P>
+static cudaError_t heur_pool_P(const HeurArgs& A, cudaStream_t s, int dev, uint64_t nwork) {
+  const int threads = hpool::NT;
+  const int rows = A.m + min(A.p - 1, A.m);
+  const size_t narg = (size_t)(A.t.n + 1) * (A.p + 1);
+  const size_t base = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
+                      ((narg + 7) & ~size_t(7)) * 2 + 32 * 4;
+  const size_t smem = base + (size_t)rows * 4 * threads;
+  cudaError_t e = set_smem((const void*)k_heur_pool<P>, smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_heur_pool<P>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  uint64_t blocks = (uint64_t)num_sms(dev) * occ;
+  const uint64_t need = (nwork + hpool::NS - 1) / hpool::NS;
+  if (blocks > need) blocks = need;
+  if (blocks < 1) blocks = 1;
+  k_heur_pool<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, int radius,
                              uint32_t r_lo, uint32_t r_hi, const int16_t* arg,
                              const int32_t* alg1_cuts, unsigned int* counter,
@@ -2036,11 +2298,21 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
   }
   A.redo = counter + 2;
   cudaError_t e;
-  switch (p) {
-    case 2: e = heur_P<2, true>(A, s, dev, R); break;
-    case 4: e = heur_P<4, true>(A, s, dev, R); break;
-    case 8: e = heur_P<8, true>(A, s, dev, R); break;
-    default: e = heur_P<16, true>(A, s, dev, R); break;
+  const char* pv = getenv("AP_HEUR_POOL");  // A/B: AP_HEUR_POOL=0 runs k_heur<P, true>
+  if (adjust_mode == 0 && !(pv && pv[0] == '0')) {
+    switch (p) {
+      case 2: e = heur_pool_P<2>(A, s, dev, R); break;
+      case 4: e = heur_pool_P<4>(A, s, dev, R); break;
+      case 8: e = heur_pool_P<8>(A, s, dev, R); break;
+      default: e = heur_pool_P<16>(A, s, dev, R); break;
+    }
+  } else {
+    switch (p) {
+      case 2: e = heur_P<2, true>(A, s, dev, R); break;
+      case 4: e = heur_P<4, true>(A, s, dev, R); break;
+      case 8: e = heur_P<8, true>(A, s, dev, R); break;
+      default: e = heur_P<16, true>(A, s, dev, R); break;
+    }
   }
   if (e != cudaSuccess) return e;
   // exact pass over the abandoned restarts (exits at once when the list is empty)

@@ -883,3 +883,34 @@ def test_memory_mode_errors(ap):
         ap.ap_plan_set_memory(plan, [-1] * 10, [0] * 10, 100)
     with pytest.raises(ap.APError):
         ap.ap_plan_set_memory(plan, [1 << 61] * 10, [0] * 10, 100)
+
+
+@pytest.mark.parametrize("p", [2, 4, 8, 16])
+def test_heuristic_pool_vs_lane_kernel_and_oracle(ap, oracle_mod, monkeypatch, p):
+    """The per-CTA simulation-pool restart kernel (k_heur_pool) and the
+    lane-per-restart kernel (AP_HEUR_POOL=0) give the oracle's winner and simulation
+    count, and every restart's own best scheme (read back through decode's per-restart
+    cache) equals the oracle's replay of that restart."""
+    import torch
+    rng = np.random.default_rng(100 + p)
+    n = int(rng.integers(max(p + 4, 2 * p), 3 * p + 20))
+    f, b, a = synth.random_tables(p, n, "b3f")
+    bw = synth.LINK_BYTES_PER_S
+    m = int(rng.integers(p, 3 * p + 2))
+    R = 3000
+    M = oracle_mod.Model(f, b, a, bw)
+    o = M.heuristic_parallel(p, m, 0x5EED, 2, 0, R, per_restart=True)
+    plan = _plan(ap, f, b, a, bw)
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    for pool in ("1", "0"):
+        monkeypatch.setenv("AP_HEUR_POOL", pool)
+        ap.ap_search_heuristic(plan, p, m, 0x5EED, 2, 0, R, 0, key)
+        torch.cuda.synchronize()
+        kv = int(key.item())
+        assert (kv >> 20, kv & 0xFFFFF) == (o["T"], o["restart"]), (pool, n, p, m)
+        assert ap.ap_last_sims() == o["sims"], pool
+        for r in [0, 1, 2, R // 2, R - 1] + [int(x) for x in rng.integers(0, R, 5)]:
+            k_r = (int(o["per_restart_T"][r]) << 20) | r
+            res = ap.ap_decode(plan, 1, p, m, seed=0x5EED, radius=2, key=k_r)
+            want = M.heuristic_restart(p, m, 0x5EED, 2, r)
+            assert res["time_ns"] == want["T"] and res["cuts"] == [int(x) for x in want["cuts"]], (pool, r)

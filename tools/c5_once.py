@@ -4,13 +4,14 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch
 import synth
 import paper_conf_cluster_liulldgl22_b200 as ap
-wl = synth.config(5)
+wl = synth.config(int(os.environ.get('AP_CFG', '5')))
+R = int(os.environ.get('AP_R', wl.restarts or 65536))
 f, b, a = wl.arrays()
 plan = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s)
 key = torch.empty(1, dtype=torch.int64, device="cuda")
 for rep in range(int(sys.argv[1]) if len(sys.argv) > 1 else 3):
     torch.cuda.synchronize(); t0 = time.perf_counter()
-    ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, wl.restarts, 0, key)
+    ap.ap_search_heuristic(plan, wl.p, wl.m, wl.seed, wl.radius, 0, R, 0, key)
     kv = int(key.item()); t1 = time.perf_counter()
     kms = ap.ap_last_kernel_ms(); sims = ap.ap_last_sims()
     res = ap.ap_decode(plan, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=kv); t2 = time.perf_counter()

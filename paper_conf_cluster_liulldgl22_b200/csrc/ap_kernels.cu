@@ -2258,7 +2258,10 @@ static cudaError_t heur_pool_P(const HeurArgs& A, cudaStream_t s, int dev, uint6
   const size_t base = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
                       ((narg + 7) & ~size_t(7)) * 2 + 32 * 4;
   const size_t smem = base + (size_t)rows * 4 * threads;
-  cudaError_t e = set_smem((const void*)k_heur_pool<P>, smem);
+  // the static slot state plus the dynamic part can pass 48 KB while the dynamic part
+  // alone does not, so the attribute is always set
+  cudaError_t e = cudaFuncSetAttribute((const void*)k_heur_pool<P>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
   if (e != cudaSuccess) return e;
   int occ = 0;
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_heur_pool<P>, threads, smem);

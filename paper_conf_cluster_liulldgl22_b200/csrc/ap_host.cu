@@ -642,7 +642,9 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   const unsigned __int128 lim = ((unsigned __int128)1 << 32) - 1;
   const int64_t a0 = (int64_t)(lim / wrow);
   const int64_t r_allow = (S >= lim) ? -1 : (int64_t)((lim - S) / wrow);
-  int want_u32 = r_allow >= (int64_t)p && r_allow >= 1;
+  // (p + 1: the offset-form sweep clamps once more before the p cool-down rows, from
+  // which a finish can sit one row's growth above S)
+  int want_u32 = r_allow >= (int64_t)p + 1;
   int clamp_first = 0, clamp_rows = 1, clamp_final = 1;
   if (want_u32) {
     auto whole = [](int64_t r) { return r >= 8 ? (r & ~int64_t(7)) : (r >= 4 ? (r & ~int64_t(3)) : r); };

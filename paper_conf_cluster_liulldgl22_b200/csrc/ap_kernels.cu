@@ -105,6 +105,41 @@ AP_DEV_INLINE void mstep(V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V wBF0,
   }
 }
 
+// Offset form of the fused steady step.  With the per-stage constants
+// c_x = wF[0] + .. + wF[x] and s_x = wF[x] + wB[x], store N_x = M_x - c_x (M_x of the
+// M-form step).  Then FF'[x] = M_{x-1} + wF[x] = N_{x-1} + c_x for x >= 1 and
+// FF'[0] = M_0 + s_0, so the next step is
+//   N'_{P-2} = max(N_{P-2} + s_{P-1}, N_{P-3}),
+//   N'_x     = max(N'_{x+1} + s_{x+1}, N_{x-1})       x = P-3 .. 1,
+//   N'_0     = max(N'_1 + s_1, N_0 + s_0):
+// P-1 fused add+max (VIADDMNMX) + 1 add per row instead of 2P-1 instructions.  N >= 0:
+// M_x >= FF[x] >= c_x, because every steady-row forward is an unsliced micro-batch whose
+// forward chain alone takes c_x.  P >= 3; state N[0..P-2].
+template <int P, typename V>
+AP_DEV_INLINE void nstep(V (&N)[P], const V (&sw)[P], uint32_t one) {
+  using O = XOps<V>;
+  static_assert(P >= 3, "");
+  V n[P];
+  n[P - 2] = O::amx(N[P - 2], sw[P - 1], N[P - 3]);
+#pragma unroll
+  for (int x = P - 3; x >= 1; --x) n[x] = O::amx(n[x + 1], sw[x + 1], N[x - 1]);
+  n[0] = O::amx(n[1], sw[1], fma_add(N[0], sw[0], one));
+#pragma unroll
+  for (int x = 0; x <= P - 2; ++x) N[x] = n[x];
+}
+
+template <int P, typename V>
+AP_DEV_INLINE void clamp_n(V (&N)[P], V S) {
+  if constexpr (sizeof(V) == 4) {
+#pragma unroll
+    for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
+  }
+}
+
+#ifndef AP_NFORM
+#define AP_NFORM 1
+#endif
+
 template <int P, typename V>
 AP_DEV_INLINE void clamp_ff(V (&FF)[P], V S) {
   if constexpr (sizeof(V) == 4) {
@@ -191,6 +226,44 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
     if (sizeof(V) == 4 && cs.first == 0) clamp_ff<P, V>(FF, S);
     int seg = (sizeof(V) == 4 && cs.first > 0) ? cs.first : cs.every;
     if (sizeof(V) != 4) seg = rem;
+    if constexpr (P >= 3 && AP_NFORM) {
+      if (rem > 0) {
+        V c[P], sw[P], N[P];
+        c[0] = wF[0];
+#pragma unroll
+        for (int x = 1; x < P; ++x) c[x] = c[x - 1] + wF[x];
+#pragma unroll
+        for (int x = 0; x < P; ++x) sw[x] = wF[x] + wB[x];
+        {  // the first step in the M-form, kept as N_x = M_x - c_x
+          V M = O::amx(FF[P - 1], wB[P - 1], FF[P - 2]);
+          N[P - 2] = M - c[P - 2];
+#pragma unroll
+          for (int x = P - 3; x >= 0; --x) {
+            M = O::amx(M, wB[x + 1], FF[x]);
+            N[x] = M - c[x];
+          }
+        }
+        int blk = (rem < seg ? rem : seg) - 1;
+        rem -= blk + 1;
+        for (;;) {
+          for (; blk >= U; blk -= U) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) nstep<P, V>(N, sw, one);
+          }
+          for (; blk > 0; --blk) nstep<P, V>(N, sw, one);
+          if (rem <= 0) break;
+          clamp_n<P, V>(N, S);
+          blk = rem < cs.every ? rem : cs.every;
+          rem -= blk;
+        }
+        // back to finishes; u32: clamped once more, so the cool-down starts <= S + W_row
+        clamp_n<P, V>(N, S);
+#pragma unroll
+        for (int x = 0; x <= P - 2; ++x) FF[x + 1] = N[x] + c[x + 1];
+        FF[0] = N[0] + c[0] + sw[0];
+      }
+      rem = 0;
+    }
     while (rem > 0) {
       int blk = rem < seg ? rem : seg;
       rem -= blk;

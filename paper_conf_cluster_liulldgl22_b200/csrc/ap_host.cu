@@ -689,6 +689,11 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   const char* sched = getenv("AP_SWEEP_SCHED");
   if (!(sched && strcmp(sched, "static") == 0)) AP_CUDA(sc.get((void**)&ctr, 16));
   AP_CUDA(g_timer.record(0, s, plan->device));
+  // one-umulhi floor(v/k) for the slice pieces when every divided value (a stage's
+  // compute total, a comm) is below 2^28 (ap_kernels.cu divk); AP_DIV1=0 disables it
+  const char* dv = getenv("AP_DIV1");
+  const int div1 = (plan->sum_f < (1ll << 28) && plan->max_comm < (1ll << 28) &&
+                    !(dv && dv[0] == '0')) ? 1 : 0;
   if (mem) {
     want_u32 = 0;  // memory mode: the generic exact kernel with the feasibility filter
     force_generic = 1;
@@ -697,7 +702,7 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
                             clamp_rows, force_generic, mem ? AP_SEARCH_FULL : mode,
                             reinterpret_cast<unsigned long long*>(key), s, &sp, rec,
                             mem ? plan->d_mem : nullptr, plan->mem_cap, ctr, clamp_first,
-                            clamp_final));
+                            clamp_final, div1));
   if (rec) {
     AP_CUDA(apk::launch_reduce2(rec, sp.blocks, reinterpret_cast<long long*>(out2), s));
     ++launches;

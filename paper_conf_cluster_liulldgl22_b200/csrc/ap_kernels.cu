@@ -43,6 +43,15 @@ AP_DEV_INLINE uint32_t divk(uint32_t v, uint32_t k, uint32_t M) {
   return q + (r >= k ? 1u : 0u);
 }
 AP_DEV_INLINE uint64_t divk(uint64_t v, uint32_t k, uint32_t) { return v / k; }
+// floor(v / k) as ONE umulhi with M = ceil(2^32/k), k >= 2: with e = M*k - 2^32 <= k-1,
+// umulhi(v, M) = floor(v/k + v*e/(k*2^32)), exact whenever v*e < 2^32, i.e. for every
+// v < 2^28 (k <= 16).  The host enables it (SweepArgs.div1) only if every stage
+// compute total and every comm is below 2^28; the table then holds the ceil magic,
+// for which divk's correction step is a no-op.
+AP_DEV_INLINE uint32_t divk(uint32_t v, uint32_t k, uint32_t M, bool div1) {
+  return div1 ? __umulhi(v, M) : divk(v, k, M);
+}
+AP_DEV_INLINE uint64_t divk(uint64_t v, uint32_t k, uint32_t, bool) { return v / k; }
 
 
 // Integer ops of the sweep, as plain operators: ptxas fuses the add of the backward
@@ -153,7 +162,7 @@ AP_DEV_INLINE void clamp_ff(V (&FF)[P], V S) {
 // memory only on the k > 1 path.
 template <int P, typename V>
 AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const V* sPf,
-                          const V* sC, uint32_t Mk, uint32_t one, V (&FF)[P]) {
+                          const V* sC, uint32_t Mk, bool div1, uint32_t one, V (&FF)[P]) {
   using O = XOps<V>;
   if (k == 1) {
     FF[0] = wF[0];
@@ -165,7 +174,7 @@ AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const 
     for (int x = 0; x < P; ++x) {
       const V Fx = sPf[c[x + 1]] - sPf[c[x]];
       const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
-      a[x] = divk(Fx, (uint32_t)k, Mk) + ((x > 0) ? divk(Cin, (uint32_t)k, Mk) : V(0));
+      a[x] = divk(Fx, (uint32_t)k, Mk, div1) + ((x > 0) ? divk(Cin, (uint32_t)k, Mk, div1) : V(0));
       al[x] = wF[x] - V(k - 1) * a[x];
       FF[x] = 0;
     }
@@ -325,10 +334,10 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
 // Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
 template <int P, typename V>
 AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const int (&c)[P + 1],
-                         const V* sPf, const V* sC, uint32_t Mk, V S, ClampSched cs,
-                         uint32_t one) {
+                         const V* sPf, const V* sC, uint32_t Mk, bool div1, V S,
+                         ClampSched cs, uint32_t one) {
   V FF[P], G[P];
-  pieces<P, V>(k, wF, c, sPf, sC, Mk, one, FF);
+  pieces<P, V>(k, wF, c, sPf, sC, Mk, div1, one, FF);
   return sweep_tail<P, V, false>(m, FF, wF, wB, S, cs, one, G);
 }
 
@@ -348,6 +357,7 @@ struct SweepArgs {
   const int64_t* mem;       // memory filter (generic kernel): [2][n+1] prefix sums
   int64_t mem_cap;
   unsigned long long* ctr;  // non-null: warp-dynamic work cursor (zeroed), chunk = ranks/lane/unit
+  int div1;                 // u32: all stage computes / comms < 2^28, one-umulhi floor(v/k)
 };
 
 AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
@@ -490,7 +500,9 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
     if (i < n) sC[i] = (V)T.comm[i];
   }
   if (threadIdx.x <= kMaxK)
-    s_mk[threadIdx.x] = (threadIdx.x <= 1) ? 0xffffffffu : (uint32_t)((1ull << 32) / threadIdx.x);
+    s_mk[threadIdx.x] = (threadIdx.x <= 1) ? 0xffffffffu
+                        : A.div1 ? (uint32_t)(((1ull << 32) + threadIdx.x - 1) / threadIdx.x)
+                                 : (uint32_t)((1ull << 32) / threadIdx.x);
   __syncthreads();
 
   const V S = (V)A.S;
@@ -590,7 +602,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
       if (live && A.mode == 0) {
         for (int k = k_lo; k <= k_hi; ++k) {
           const uint32_t Mk = s_mk[k];
-          const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, S, cs, A.one);
+          const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, A.div1 != 0, S, cs, A.one);
           if (Tc < bestT) {
             bestT = Tc;
             bestIdx = base + (uint64_t)(k - k_lo);
@@ -615,7 +627,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
           V Tc;
           if constexpr (P >= 2) {
             V FF[P];
-            pieces<P, V>(k, wF, c, sPf, sC, s_mk[k], A.one, FF);
+            pieces<P, V>(k, wF, c, sPf, sC, s_mk[k], A.div1 != 0, A.one, FF);
             Tc = FF[0] + G[0];
 #pragma unroll
             for (int x = 1; x < P; ++x) {
@@ -623,7 +635,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
               Tc = v > Tc ? v : Tc;
             }
           } else {
-            Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, s_mk[k], S, cs, A.one);
+            Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, s_mk[k], A.div1 != 0, S, cs, A.one);
           }
           if (Tc < bestT) {
             bestT = Tc;
@@ -2281,12 +2293,13 @@ cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, u
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
                          SweepPlan* sp, unsigned long long* rec, const int64_t* mem,
                          int64_t mem_cap, unsigned long long* ctr, int clamp_first,
-                         int clamp_final) {
+                         int clamp_final, int div1) {
   int dev = 0;
   cudaGetDevice(&dev);
   SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key,
               clamp_rows < 1 ? 1 : clamp_rows, clamp_first < 0 ? 0 : clamp_first,
-              clamp_first < 0 ? 1 : clamp_final, 1u, mode, rec, mem, mem_cap, ctr};
+              clamp_first < 0 ? 1 : clamp_final, 1u, mode, rec, mem, mem_cap, ctr,
+              want_u32 ? div1 : 0};
   const bool exact = !mem && has_exact(p) && m >= p && (!force_generic || mode != 0);
   sp->exact_p = exact ? 1 : 0;
   sp->fast_u32 = (exact && want_u32) ? 1 : 0;

@@ -51,7 +51,7 @@ cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, u
                          SweepPlan* plan_out, unsigned long long* rec = nullptr,
                          const int64_t* mem = nullptr, int64_t mem_cap = 0,
                          unsigned long long* ctr = nullptr, int clamp_first = -1,
-                         int clamp_final = 1);
+                         int clamp_final = 1, int div1 = 0);
 
 // Two-phase reduction (NEXT N3).  With `rec` (u64[2 * sweep_max_blocks(dev)]) passed
 // to launch_sweep, each CTA stores its lexicographic min (T, index) there instead of

@@ -914,3 +914,35 @@ def test_heuristic_pool_vs_lane_kernel_and_oracle(ap, oracle_mod, monkeypatch, p
             res = ap.ap_decode(plan, 1, p, m, seed=0x5EED, radius=2, key=k_r)
             want = M.heuristic_restart(p, m, 0x5EED, 2, r)
             assert res["time_ns"] == want["T"] and res["cuts"] == [int(x) for x in want["cuts"]], (pool, r)
+
+
+def test_exhaustive_div1_pieces(ap, oracle_mod, monkeypatch):
+    """The one-umulhi floor(v/k) of the slice pieces (values < 2^28) and the corrected
+    two-step form (AP_DIV1=0) give the same key as the oracle's argmin, on C2 (k 1..4)
+    and on random tables with values just below the 2^28 bound."""
+    import torch
+    cases = []
+    wl = synth.config(2)
+    cases.append((*wl.arrays(), wl.link_bytes_per_s, wl.p, wl.m, 1, 4))
+    rng = np.random.default_rng(77)
+    for t in range(4):
+        n = int(rng.integers(6, 12))
+        f = rng.integers((1 << 28) // (2 * n), (1 << 28) // n, n).astype(np.int64)
+        b = rng.integers(0, 1 << 20, n).astype(np.int64)
+        a = rng.integers(0, 1 << 27, n).astype(np.int64)
+        p = int(rng.integers(2, min(n, 8) + 1))
+        cases.append((f, b, a, 10**9, p, int(rng.integers(p, p + 6)), 1, 16))
+    key = torch.empty(1, dtype=torch.int64, device="cuda")
+    for f, b, a, bw, p, m, k_lo, k_hi in cases:
+        plan = _plan(ap, f, b, a, bw)
+        N = ap.ap_count(len(f), p)
+        keys = []
+        for d in ("1", "0"):
+            monkeypatch.setenv("AP_DIV1", d)
+            ap.ap_search_exhaustive(plan, p, m, k_lo, k_hi, 0, N, key)
+            torch.cuda.synchronize()
+            keys.append(int(key.item()))
+        assert keys[0] == keys[1]
+        o = oracle_mod.Model(f, b, a, bw).exhaustive(p, m, k_lo, k_hi)
+        res = ap.ap_decode(plan, 0, p, m, k_lo, k_hi, key=keys[0])
+        assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])

@@ -1583,10 +1583,11 @@ __global__ void __launch_bounds__(hpool::NT, 2) k_heur_pool(HeurArgs A) {
           }
         }
       }
-      if (st == 0 && !s_stop) {
+      // s_stop is written and read by several slot threads in the same phase: atomics
+      if (st == 0 && atomicAdd(&s_stop, 0) == 0) {
         const uint32_t r = atomicAdd(A.counter, 1u) + A.r_lo;
         if (r >= A.r_hi) {
-          s_stop = 1;
+          atomicOr(&s_stop, 1);
         } else {
           // restart start: Alg. 1 (r = 0) or the seeded perturbation (reading Q21)
           int prev = 0;

@@ -642,8 +642,8 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   const unsigned __int128 lim = ((unsigned __int128)1 << 32) - 1;
   const int64_t a0 = (int64_t)(lim / wrow);
   const int64_t r_allow = (S >= lim) ? -1 : (int64_t)((lim - S) / wrow);
-  // (p + 1: the offset-form sweep clamps once more before the p cool-down rows, from
-  // which a finish can sit one row's growth above S)
+  // (p + 1: after a clamp the offset-form sweep's conversion back to finishes can sit
+  // one row's growth above S before the p cool-down rows)
   int want_u32 = r_allow >= (int64_t)p + 1;
   int clamp_first = 0, clamp_rows = 1, clamp_final = 1;
   if (want_u32) {
@@ -666,7 +666,9 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
         clamp_final = 1;
       } else {
         const int64_t last = L - every * ((L - 1) / every);
-        clamp_final = (last + p > r_allow) ? 1 : 0;
+        // + 1: the offset-form sweep converts N back to finishes (FF = N + c) before the
+        // p cool-down rows, one more row of growth
+        clamp_final = (last + p + 1 > r_allow) ? 1 : 0;
       }
     }
   }

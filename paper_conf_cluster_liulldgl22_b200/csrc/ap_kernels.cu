@@ -167,7 +167,7 @@ AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const 
   if (k == 1) {
     FF[0] = wF[0];
 #pragma unroll
-    for (int x = 1; x < P; ++x) FF[x] = O::ad(FF[x - 1], wF[x], one);
+    for (int x = 1; x < P; ++x) FF[x] = fma_add(FF[x - 1], wF[x], one);  // FMA pipe: ALU-bound
   } else {
     V a[P], al[P];
 #pragma unroll
@@ -237,12 +237,13 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
     if (sizeof(V) != 4) seg = rem;
     if constexpr (P >= 3 && AP_NFORM) {
       if (rem > 0) {
+        // (adds outside the max chain go to the FMA pipe: the kernel is ALU-bound)
         V c[P], sw[P], N[P];
         c[0] = wF[0];
 #pragma unroll
-        for (int x = 1; x < P; ++x) c[x] = c[x - 1] + wF[x];
+        for (int x = 1; x < P; ++x) c[x] = fma_add(c[x - 1], wF[x], one);
 #pragma unroll
-        for (int x = 0; x < P; ++x) sw[x] = wF[x] + wB[x];
+        for (int x = 0; x < P; ++x) sw[x] = fma_add(wF[x], wB[x], one);
         {  // the first step in the M-form, kept as N_x = M_x - c_x
           V M = O::amx(FF[P - 1], wB[P - 1], FF[P - 2]);
           N[P - 2] = M - c[P - 2];
@@ -265,11 +266,12 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
           blk = rem < cs.every ? rem : cs.every;
           rem -= blk;
         }
-        // back to finishes; u32: clamped once more, so the cool-down starts <= S + W_row
-        clamp_n<P, V>(N, S);
+        // back to finishes (u32: FF = N + c sits up to one row's growth above N, which
+        // the host's clamp_final test allows for: last segment + 1 + p rows)
+        if (cs.fin) clamp_n<P, V>(N, S);
 #pragma unroll
-        for (int x = 0; x <= P - 2; ++x) FF[x + 1] = N[x] + c[x + 1];
-        FF[0] = N[0] + c[0] + sw[0];
+        for (int x = 0; x <= P - 2; ++x) FF[x + 1] = fma_add(N[x], c[x + 1], one);
+        FF[0] = fma_add(N[0], fma_add(c[0], sw[0], one), one);
       }
       rem = 0;
     }

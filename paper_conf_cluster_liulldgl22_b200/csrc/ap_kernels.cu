@@ -1071,63 +1071,52 @@ AP_DEV_INLINE uint32_t sim_fast_bits(int m, const uint32_t (&wF)[P], const uint3
   return b;
 }
 
-// backtrack_master (ap_device.cuh) specialised to the fast path: p == P, k == 1,
-// m >= P (so w_x = P-1-x, W0 = P-1), m <= 32767.  The same walk and the same reading
-// (O5 tie rule, O6 master = most 1F1B-phase path ops, ties -> higher stage, none ->
-// P-1), but the per-stage counts live in registers: the path stays on one stage for
-// a run of ops, so a run counter is flushed into 16-bit fields of NW words only when
-// the path changes stage (unrolled select, no local memory).
-template <int P>
-AP_DEV_INLINE int backtrack_master_fast(int m, BitsRef br) {
-  constexpr int NW = (P + 1) / 2;
+// backtrack_master (ap_device.cuh) specialised to the fast path (p == P, k == 1,
+// m >= P, so w_x = P-1-x, W0 = P-1; m <= 32767) and written without divergent
+// branches: each op's move is computed with selects, so the lanes of a warp only part
+// at the loop exit (C5 pool kernel 1.68 -> 1.19 ms).  Same walk and reading (O5 tie rule, O6 master; the 1F1B phase of stage x is
+// rows [P-1, m-1+x] for both F and B).  Per-stage counts are CB-bit fields of NW
+// registers (CB = 8 needs 2m <= 255), flushed when the path changes stage.
+template <int P, int CB>
+AP_DEV_INLINE int backtrack_master_bl(int m, BitsRef br) {
+  constexpr int PER = 32 / CB;
+  constexpr int NW = (P + PER - 1) / PER;
   uint32_t cw[NW];
 #pragma unroll
   for (int w = 0; w < NW; ++w) cw[w] = 0;
-  auto flush = [&](int x, uint32_t run) {
-    const uint32_t inc = run << (16 * (x & 1));
-#pragma unroll
-    for (int w = 0; w < NW; ++w) cw[w] += (w == (x >> 1)) ? inc : 0u;
-  };
-  int kind = 1, x = 0, j = m - 1;
+  int x = 0, row = m + P - 2;  // the sink B(0, m-1)
+  bool onB = true;
   uint32_t run = 0;
   for (;;) {
-    const int wx = P - 1 - x;
-    const int row = kind ? (j + P - 1) : (j + x);
     const uint32_t word = br.base[(size_t)row * br.stride];
-    run += kind ? (j < m - wx ? 1u : 0u) : (j >= wx ? 1u : 0u);
-    if (kind == 0 && j == 0 && x == 0) break;  // the source F(0, 0)
-    const bool cross = kind ? (x < P - 1 && ((word >> (x + 16)) & 1u))
-                            : (x > 0 && (j == 0 || ((word >> x) & 1u)));
-    if (cross) {
-      flush(x, run);
+    run += (row >= P - 1 && row <= m - 1 + x) ? 1u : 0u;
+    if (!onB && row == 0) break;  // the source F(0, 0)
+    const bool cB = onB && x < P - 1 && ((word >> (x + 16)) & 1u);
+    const bool cF = !onB && x > 0 && (row == x || ((word >> x) & 1u));
+    if (cB || cF) {
+      const uint32_t inc = run << (CB * (x % PER));
+#pragma unroll
+      for (int w = 0; w < NW; ++w) cw[w] += (w == x / PER) ? inc : 0u;
       run = 0;
-      x += kind ? 1 : -1;
-      continue;
     }
-    if (kind) {
-      const int jf = j + wx;
-      if (jf <= m - 1) {  // F(x, y + w_x) just before it in the same row
-        kind = 0;
-        j = jf;
-      } else if (j >= 1) {  // previous BP of the stage
-        j = j - 1;
-      } else {  // w_x = m cannot happen here (m >= P > w_x); kept for symmetry
-        kind = 0;
-        j = m - 1;
-      }
-    } else if (j > wx) {  // 1F1B: the previous op is B(x, j - w_x - 1)
-      kind = 1;
-      j = j - wx - 1;
-    } else {  // warm-up: F(x, j-1)
-      j = j - 1;
-    }
+    const bool Fhere = row <= m - 1 + x;  // F(x) exists in this row
+    const int r0 = row;
+    row = onB ? ((cB || Fhere) ? r0 : r0 - 1) : r0 - 1;
+    const bool nB = onB ? (cB || !Fhere) : (!cF && r0 > P - 1);
+    x += (cB ? 1 : 0) - (cF ? 1 : 0);
+    onB = nB;
   }
-  flush(x, run);
+  {
+    const uint32_t inc = run << (CB * (x % PER));
+#pragma unroll
+    for (int w = 0; w < NW; ++w) cw[w] += (w == x / PER) ? inc : 0u;
+  }
+  constexpr uint32_t MASK = (CB == 8) ? 0xffu : 0xffffu;
   int best = P - 1;
-  uint32_t bc = (cw[(P - 1) >> 1] >> (16 * ((P - 1) & 1))) & 0xffffu;
+  uint32_t bc = (cw[(P - 1) / PER] >> (CB * ((P - 1) % PER))) & MASK;
 #pragma unroll
   for (int xx = P - 2; xx >= 0; --xx) {
-    const uint32_t c = (cw[xx >> 1] >> (16 * (xx & 1))) & 0xffffu;
+    const uint32_t c = (cw[xx / PER] >> (CB * (xx % PER))) & MASK;
     if (c > bc) {
       best = xx;
       bc = c;
@@ -1336,7 +1325,7 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
     }
     int Mc;
     if constexpr (FAST) {
-      Mc = backtrack_master_fast<P>(m, br);
+      Mc = m <= 127 ? backtrack_master_bl<P, 8>(m, br) : backtrack_master_bl<P, 16>(m, br);
     } else {
       int len;
       Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
@@ -1639,7 +1628,8 @@ __global__ void __launch_bounds__(hpool::NT, 2) k_heur_pool(HeurArgs A) {
         s_aband[s] = 1;
       } else {
         s_chT[s][idx] = t32;
-        s_chM[s][idx] = (int8_t)backtrack_master_fast<P>(m, br);
+        s_chM[s][idx] = (int8_t)(m <= 127 ? backtrack_master_bl<P, 8>(m, br)
+                                          : backtrack_master_bl<P, 16>(m, br));
       }
       atomicSub(&s_pend[s], 1);
     }

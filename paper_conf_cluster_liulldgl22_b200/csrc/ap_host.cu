@@ -764,6 +764,28 @@ ap_status ap_key2_select(const int64_t* local, const int64_t* t_star, int64_t* i
   return AP_OK;
 }
 
+// u32 fast path of the restart kernels: every value grows by at most
+// W_row per row and is clamped to S every CR rows (the cool-down adds p more rows), so
+// S = 2^32-1 - (max(CR,p)+1)*W_row keeps everything exact below S; 0 = no fast path.
+// Test overrides: AP_HEUR=int64 disables it; AP_HEUR_S=<v> lowers the bound so that
+// simulations saturate and exercise the exact fallbacks.
+static uint32_t heur_fast_bound(const ap_plan* plan, int p, int CR) {
+  const unsigned __int128 hw = (unsigned __int128)(plan->sum_f + plan->sum_b) +
+                               (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
+  const unsigned __int128 span = hw * (unsigned __int128)((CR > p ? CR : p) + 1);
+  const unsigned __int128 lim32 = ((unsigned __int128)1 << 32) - 1;
+  uint32_t fastS = 0;
+  if (span < lim32) fastS = (uint32_t)(lim32 - span);
+  const char* hov = getenv("AP_HEUR");
+  if (hov && strcmp(hov, "int64") == 0) fastS = 0;
+  const char* hs = getenv("AP_HEUR_S");
+  if (hs && fastS > 0) {
+    const unsigned long long v = strtoull(hs, nullptr, 10);
+    if (v > 0 && v < fastS) fastS = (uint32_t)v;
+  }
+  return fastS;
+}
+
 ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
                               int32_t radius, uint32_t r_lo, uint32_t r_hi, int32_t adjust_mode,
                               int64_t* key, ap_stream_t stream) {
@@ -799,25 +821,8 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
     g_hcache.cap = need;
     g_hcache.dev = plan->device;
   }
-  // u32 fast path: every value grows by at most W_row per row and
-  // is clamped to S every CR rows (the cool-down adds p more rows), so
-  // S = 2^32-1 - (max(CR,p)+1)*W_row keeps everything exact below S.
   const int hCR = 32;
-  const unsigned __int128 hw = (unsigned __int128)(plan->sum_f + plan->sum_b) +
-                               (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
-  const unsigned __int128 span = hw * (unsigned __int128)((hCR > p ? hCR : p) + 1);
-  const unsigned __int128 lim32 = ((unsigned __int128)1 << 32) - 1;
-  uint32_t fastS = 0;
-  if (span < lim32) fastS = (uint32_t)(lim32 - span);
-  // test overrides: AP_HEUR=int64 disables the u32 pass; AP_HEUR_S=<v> lowers its
-  // bound so that restarts saturate and exercise the exact redo pass
-  const char* hov = getenv("AP_HEUR");
-  if (hov && strcmp(hov, "int64") == 0) fastS = 0;
-  const char* hs = getenv("AP_HEUR_S");
-  if (hs && fastS > 0) {
-    const unsigned long long v = strtoull(hs, nullptr, 10);
-    if (v > 0 && v < fastS) fastS = (uint32_t)v;
-  }
+  const uint32_t fastS = heur_fast_bound(plan, p, hCR);
   AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), d_ctr, s));
   AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_heuristic(plan->dev(), p, m, seed, radius, r_lo, r_hi, d_arg, d_a1, d_ctr,
@@ -872,7 +877,7 @@ ap_status ap_search_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_
   AP_CUDA(g_timer.record(0, s, plan->device));
   AP_CUDA(apk::launch_reach(plan->dev(), p, m, seed, radius, r_lo, r_hi, vmax, d_arg, d_a1, d_ctr,
                             reinterpret_cast<unsigned long long*>(key), d_sims, nullptr, d_scr,
-                            s));
+                            s, heur_fast_bound(plan, p, 32)));
   AP_CUDA(g_timer.record(1, s, plan->device));
   g_timer.sims_on_device = true;
   g_timer.truncated_valid = true;

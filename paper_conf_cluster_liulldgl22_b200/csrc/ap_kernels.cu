@@ -1672,6 +1672,8 @@ struct ReachArgs {
   uint32_t* g_queue;          // [quads][vmax]: node | master << 24
   unsigned long long* stats;  // optional: [0] simulations, [1] truncated restarts
   int32_t* replay;            // optional: best cuts of the (single) restart
+  uint32_t S;                 // > 0: u32 fast simulation below S (as k_heur_pool), int64
+                              // sim_exact for a simulation that reaches S
 };
 
 AP_DEV_INLINE uint32_t cut_hash(const int (&c)[33], int p) {
@@ -1822,12 +1824,32 @@ __global__ void __launch_bounds__(128) k_reach(ReachArgs A) {
       for (int x = 0; x <= P; ++x) cc[x] = (x <= p) ? cand[x] : n;
       int64_t F[P], B[P], C[P];
       stage_costs<P>(T, p, cc, F, B, C);
-      uint32_t pb[P];
+      bool exact = true;
+      if constexpr (P >= 2 && P <= 16) {
+        // u32 fast path (p == P, m >= P): T below S is exact; at S recompute in int64
+        if (A.S > 0 && p == P && m >= P && m <= 32767) {
+          uint32_t wF[P], wB[P];
 #pragma unroll
-      for (int x = 0; x < P; ++x) pb[x] = 0;
-      Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
-      int len;
-      Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+          for (int x = 0; x < P; ++x) {
+            wF[x] = (uint32_t)(F[x] + ((x > 0) ? C[x - 1] : 0));
+            wB[x] = (uint32_t)(B[x] + C[x]);
+          }
+          const uint32_t t32 = sim_fast_bits<P>(m, wF, wB, A.S, 32, br);
+          if (t32 < A.S) {
+            Tc = (int64_t)t32;
+            Mc = m <= 127 ? backtrack_master_bl<P, 8>(m, br) : backtrack_master_bl<P, 16>(m, br);
+            exact = false;
+          }
+        }
+      }
+      if (exact) {
+        uint32_t pb[P];
+#pragma unroll
+        for (int x = 0; x < P; ++x) pb[x] = 0;
+        Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
+        int len;
+        Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+      }
       for (int x = 1; x <= p - 1; ++x) Qc[(size_t)slot * P + (x - 1)] = (int16_t)cand[x];
       Qh[slot] = cut_hash(cand, p);
     }
@@ -2466,10 +2488,11 @@ cudaError_t launch_reach(const DevTables& t, int p, int m, uint64_t seed, int ra
                          uint32_t r_lo, uint32_t r_hi, int vmax, const int16_t* arg,
                          const int32_t* alg1_cuts, unsigned int* counter,
                          unsigned long long* key, unsigned long long* stats, int32_t* replay,
-                         void* scratch, cudaStream_t s) {
+                         void* scratch, cudaStream_t s, uint32_t fastS) {
   int dev = 0;
   cudaGetDevice(&dev);
   ReachArgs A{};
+  A.S = fastS;
   A.t = t;
   A.p = p;
   A.m = m;

@@ -99,7 +99,7 @@ cudaError_t launch_reach(const DevTables& t, int p, int m, uint64_t seed, int ra
                          uint32_t r_lo, uint32_t r_hi, int vmax, const int16_t* arg,
                          const int32_t* alg1_cuts, unsigned int* counter,
                          unsigned long long* key, unsigned long long* stats, int32_t* replay,
-                         void* scratch, cudaStream_t s);
+                         void* scratch, cudaStream_t s, uint32_t fastS = 0);
 
 // Decode helper: unrank lex rank -> cut vector int32[p-1].
 cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,

@@ -946,3 +946,29 @@ def test_exhaustive_div1_pieces(ap, oracle_mod, monkeypatch):
         o = oracle_mod.Model(f, b, a, bw).exhaustive(p, m, k_lo, k_hi)
         res = ap.ap_decode(plan, 0, p, m, k_lo, k_hi, key=keys[0])
         assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+
+
+@pytest.mark.parametrize("mode", ["fast", "int64", "saturating"])
+def test_reach_fast_and_exact_simulation(ap, oracle_mod, monkeypatch, mode):
+    """The reachable-set kernel's u32 fast simulation (p in {2,4,8,16}, m >= p), the
+    exact int64 one (AP_HEUR=int64) and the fast one with a bound so low that many
+    simulations fall back to int64 (AP_HEUR_S) all give the oracle's winner,
+    simulation count and truncations."""
+    if mode == "int64":
+        monkeypatch.setenv("AP_HEUR", "int64")
+    rng = np.random.default_rng(61)
+    for trial, p in enumerate((2, 4, 8, 16)):
+        n = int(rng.integers(p + 6, 3 * p + 20))
+        f, b, a = synth.random_tables(900 + trial, n, "b3f")
+        bw = synth.LINK_BYTES_PER_S
+        M = oracle_mod.Model(f, b, a, bw)
+        m = int(rng.integers(p, 3 * p + 2))
+        R = 300
+        o = M.reach_parallel(p, m, 0x5EED, 2, 0, R, vmax=1024)
+        if mode == "saturating":
+            monkeypatch.setenv("AP_HEUR_S", str(int(o["T"]) + 1))
+        plan = _plan(ap, f, b, a, bw)
+        key, sims, trunc = _reach(ap, plan, p, m, 0x5EED, 2, 0, R, 1024)
+        assert (key >> 20, key & 0xFFFFF, sims, trunc) == (o["T"], o["restart"], o["sims"], o["truncated"]), (mode, p)
+        res = ap.ap_decode_reachable(plan, p, m, 0x5EED, 2, 1024, key)
+        assert res["time_ns"] == o["T"] and res["cuts"] == [int(x) for x in o["cuts"]]

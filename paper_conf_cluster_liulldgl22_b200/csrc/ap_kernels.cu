@@ -1674,6 +1674,8 @@ struct ReachArgs {
   int32_t* replay;            // optional: best cuts of the (single) restart
   uint32_t S;                 // > 0: u32 fast simulation below S (as k_heur_pool), int64
                               // sim_exact for a simulation that reaches S
+  uint32_t* g_tab;            // pool: per-list open-addressing table [lists][tab_size] of
+  int tab_size;               //   (restart tag << 11 | node), zeroed per search
 };
 
 AP_DEV_INLINE uint32_t cut_hash(const int (&c)[33], int p) {
@@ -1934,6 +1936,272 @@ struct CpathArgs {
   int64_t* finP;
   int* order;  // path scratch: encoded ops sink -> source
 };
+
+// ---------------------------------------------------------------------------
+// K3r as a simulation pool (DESIGN.md R-N1, §5.5): the reachable-set search of k_reach,
+// restructured like k_heur_pool.  A CTA owns NS restart slots; each slot's evaluated
+// list (cuts, hash) and FIFO queue live in global scratch (per-slot, L1/L2-resident).
+//   phase A, one thread per slot: fold the finished children of the node it expanded
+//     into the evaluated list in child order (new ones only, up to vmax: the
+//     truncation point of k_reach and the oracle), queue those with master <= i,
+//     then pop the next queued scheme with master > 0 and emit its children as jobs;
+//   phase B, one job per thread: drop the child if it is already evaluated (hash scan
+//     + compare over the slot's list), else simulate it (u32 fast path with an
+//     in-lane int64 fallback at the bound, as k_reach).
+// Siblings a, a', b, b' are pairwise distinct, so deduplicating each child against the
+// list as it stood before the expansion is the serial order's result.
+constexpr int RP_NT = 256, RP_NS = 96, RP_RING = 512;
+
+AP_DEV_INLINE uint32_t cut_hash16(const int16_t* c, int p) {
+  uint32_t h = 0x811c9dc5u;
+  for (int x = 1; x <= p - 1; ++x) h = (h ^ (uint32_t)(int)c[x]) * 0x01000193u;
+  return h;
+}
+
+template <int P>
+__global__ void __launch_bounds__(RP_NT, 2) k_reach_pool(ReachArgs A) {
+  constexpr int NT = RP_NT, NS = RP_NS, RING = RP_RING;
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int n = A.t.n, p = A.p, m = A.m, P1 = p + 1, vmax = A.vmax;
+  int16_t* s_arg = reinterpret_cast<int16_t*>(smem + ((used + 15) & ~size_t(15)));
+  const int narg = (n + 1) * P1;
+  int32_t* s_a1 = reinterpret_cast<int32_t*>(s_arg + ((narg + 7) & ~7));
+  uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_a1 + 32);
+  __shared__ int16_t s_cuts[NS][5][P + 1];  // [0] node being expanded, [1+idx] child idx
+  __shared__ int64_t s_chT[NS][4], s_bestT[NS];
+  __shared__ int8_t s_chM[NS][4], s_chDup[NS][4];
+  __shared__ uint32_t s_r[NS];
+  __shared__ int s_pend[NS], s_nv[NS], s_qh[NS], s_qt[NS], s_best[NS], s_nsims[NS];
+  __shared__ int8_t s_state[NS], s_parM[NS], s_valid[NS];
+  __shared__ uint16_t s_ring[RING];
+  __shared__ int s_head, s_tail, s_stop;
+  const int tid = threadIdx.x;
+  for (int e = tid; e < narg; e += NT) s_arg[e] = A.arg[e];
+  for (int e = tid; e < p - 1; e += NT) s_a1[e] = A.alg1[e];
+  for (int q = tid; q < NS; q += NT) s_state[q] = 0;
+  if (tid == 0) {
+    s_head = 0;
+    s_tail = 0;
+    s_stop = 0;
+  }
+  __syncthreads();
+  const BitsRef br{s_bits + tid, NT};
+  TimesRef not_{nullptr, nullptr, nullptr};
+  unsigned long long my_key = 0x7fffffffffffffffull, my_sims = 0, my_trunc = 0;
+
+  for (;;) {
+    // ---- phase A: fold results, expand the next queued scheme, refill free slots
+    if (tid < NS) {
+      const int s = tid;
+      const size_t L = (size_t)blockIdx.x * NS + s;  // this slot's global lists
+      int16_t* Qc = A.g_cuts + L * (size_t)vmax * P;
+      uint32_t* Qh = A.g_hash + L * (size_t)vmax;
+      uint32_t* Qq = A.g_queue + L * (size_t)vmax;
+      int st = s_state[s];
+      if (st != 0 && s_pend[s] == 0) {
+        int nv = s_nv[s], qh = s_qh[s], qt = s_qt[s], best = s_best[s], nsims = s_nsims[s];
+        int64_t bestT = s_bestT[s];
+        bool trunc = false;
+        uint32_t* Tb = A.g_tab + L * (size_t)A.tab_size;
+        const uint32_t tag = (s_r[s] + 1u) & 0x1fffffu;
+        auto insert = [&](uint32_t h, int node) {  // linear probing; other tags = empty
+          uint32_t pos = h & (uint32_t)(A.tab_size - 1);
+          while ((Tb[pos] >> 11) == tag) pos = (pos + 1) & (uint32_t)(A.tab_size - 1);
+          Tb[pos] = (tag << 11) | (uint32_t)node;
+        };
+        if (st == 1) {  // the start was simulated: it is node 0
+          for (int x = 1; x <= p - 1; ++x) Qc[x - 1] = s_cuts[s][1][x];
+          Qh[0] = cut_hash16(s_cuts[s][1], p);
+          insert(Qh[0], 0);
+          Qq[0] = (uint32_t)s_chM[s][0] << 24;
+          nv = 1;
+          qh = 0;
+          qt = 1;
+          best = 0;
+          bestT = s_chT[s][0];
+          nsims = 1;
+        } else {  // children of the expanded node, in child order
+          const int valid = s_valid[s], i = s_parM[s];
+          for (int idx = 0; idx < 4 && !trunc; ++idx) {
+            if (!((valid >> idx) & 1) || s_chDup[s][idx]) continue;
+            if (nv >= vmax) {
+              trunc = true;
+              break;
+            }
+            for (int x = 1; x <= p - 1; ++x) Qc[(size_t)nv * P + (x - 1)] = s_cuts[s][1 + idx][x];
+            Qh[nv] = cut_hash16(s_cuts[s][1 + idx], p);
+            insert(Qh[nv], nv);
+            ++nsims;
+            const int64_t Tc = s_chT[s][idx];
+            const int Mc = s_chM[s][idx];
+            if (Tc < bestT) {
+              bestT = Tc;
+              best = nv;
+            }
+            if (Mc <= i) Qq[qt++] = (uint32_t)nv | ((uint32_t)Mc << 24);
+            ++nv;
+          }
+        }
+        // pop queued schemes (master-0 ones are not expanded) until one has children
+        int valid = 0, nj = 0;
+        while (!trunc && nj == 0 && qh < qt) {
+          const uint32_t e = Qq[qh++];
+          const int i = (int)(e >> 24);
+          if (i == 0) continue;
+          const int u = (int)(e & 0xffffffu);
+          int16_t* cur = s_cuts[s][0];
+          cur[0] = 0;
+          cur[p] = (int16_t)n;
+          for (int x = 1; x <= p - 1; ++x) cur[x] = Qc[(size_t)u * P + (x - 1)];
+          for (int idx = 0; idx < 4; ++idx)
+            if (pool_child(cur, idx, i, p, P1, s_arg, s_cuts[s][1 + idx])) {
+              valid |= 1 << idx;
+              ++nj;
+            }
+          s_parM[s] = (int8_t)i;
+        }
+        if (nj > 0) {
+          const int at = atomicAdd(&s_tail, nj);
+          int q = 0;
+          for (int idx = 0; idx < 4; ++idx)
+            if ((valid >> idx) & 1) s_ring[(at + q++) & (RING - 1)] = (uint16_t)(s * 4 + idx);
+          s_pend[s] = nj;
+          s_valid[s] = (int8_t)valid;
+          s_nv[s] = nv;
+          s_qh[s] = qh;
+          s_qt[s] = qt;
+          s_best[s] = best;
+          s_bestT[s] = bestT;
+          s_nsims[s] = nsims;
+          st = 2;
+        } else {  // queue exhausted or vmax reached: the restart is finished
+          my_sims += (unsigned long long)nsims;
+          my_trunc += trunc ? 1 : 0;
+          if (bestT < (1ll << 43))
+            my_key = min(my_key, ((unsigned long long)bestT << 20) | s_r[s]);
+          st = 0;
+        }
+      }
+      if (st == 0 && atomicAdd(&s_stop, 0) == 0) {
+        const uint32_t r = atomicAdd(A.counter, 1u) + A.r_lo;
+        if (r >= A.r_hi) {
+          atomicOr(&s_stop, 1);
+        } else {
+          // restart start: Alg. 1 (r = 0) or the seeded perturbation (reading Q21)
+          int prev = 0;
+          int16_t* c = s_cuts[s][1];
+          c[0] = 0;
+          c[p] = (int16_t)n;
+          for (int x = 1; x <= p - 1; ++x) {
+            int64_t v = s_a1[x - 1];
+            if (r != 0) {
+              const uint64_t u = splitmix64(A.seed ^ ((uint64_t)r << 32) ^ (uint64_t)x);
+              v += (int64_t)(u % (uint64_t)(2 * A.radius + 1)) - A.radius;
+              v = v < prev + 1 ? prev + 1 : v;
+              v = v > n - (p - x) ? n - (p - x) : v;
+            }
+            c[x] = (int16_t)v;
+            prev = (int)v;
+          }
+          s_r[s] = r;
+          s_nv[s] = 0;  // the start is simulated without a duplicate check
+          s_pend[s] = 1;
+          const int at = atomicAdd(&s_tail, 1);
+          s_ring[at & (RING - 1)] = (uint16_t)(s * 4);
+          st = 1;
+        }
+      }
+      s_state[s] = (int8_t)st;
+    }
+    if (!__syncthreads_or(tid < NS && s_state[tid] != 0)) break;
+    // ---- phase B: one queued child per thread
+    const int head = s_head;
+    const int nj = min(s_tail - head, NT);
+    if (tid < nj) {
+      const int job = s_ring[(head + tid) & (RING - 1)];
+      const int s = job >> 2, idx = job & 3;
+      const int16_t* cr = s_cuts[s][1 + idx];
+      // already evaluated?  (the list as it stood before this expansion)
+      bool dup = false;
+      const int nv = s_nv[s];
+      if (nv > 0) {
+        const size_t L = (size_t)blockIdx.x * NS + s;
+        const int16_t* Qc = A.g_cuts + L * (size_t)vmax * P;
+        const uint32_t* Qh = A.g_hash + L * (size_t)vmax;
+        const uint32_t* Tb = A.g_tab + L * (size_t)A.tab_size;
+        const uint32_t tag = (s_r[s] + 1u) & 0x1fffffu;
+        const uint32_t h = cut_hash16(cr, p);
+        for (uint32_t pos = h & (uint32_t)(A.tab_size - 1);; pos = (pos + 1) & (uint32_t)(A.tab_size - 1)) {
+          const uint32_t e = Tb[pos];
+          if ((e >> 11) != tag) break;  // empty for this restart: not evaluated
+          const int j = (int)(e & 0x7ffu);
+          if (Qh[j] != h) continue;
+          bool same = true;
+          for (int x = 1; x <= p - 1; ++x) same = same && (Qc[(size_t)j * P + (x - 1)] == cr[x]);
+          if (same) {
+            dup = true;
+            break;
+          }
+        }
+      }
+      s_chDup[s][idx] = dup ? 1 : 0;
+      if (!dup) {
+        int cc[P + 1];
+#pragma unroll
+        for (int x = 0; x <= P; ++x) cc[x] = (x <= p) ? (int)cr[x] : n;
+        int64_t F[P], B[P], C[P];
+        stage_costs<P>(T, p, cc, F, B, C);
+        int64_t Tc = 0;
+        int Mc = 0;
+        bool exact = true;
+        if constexpr (P >= 2 && P <= 16) {
+          if (A.S > 0 && p == P && m >= P && m <= 32767) {
+            uint32_t wF[P], wB[P];
+#pragma unroll
+            for (int x = 0; x < P; ++x) {
+              wF[x] = (uint32_t)(F[x] + ((x > 0) ? C[x - 1] : 0));
+              wB[x] = (uint32_t)(B[x] + C[x]);
+            }
+            const uint32_t t32 = sim_fast_bits<P>(m, wF, wB, A.S, 32, br);
+            if (t32 < A.S) {
+              Tc = (int64_t)t32;
+              Mc = m <= 127 ? backtrack_master_bl<P, 8>(m, br) : backtrack_master_bl<P, 16>(m, br);
+              exact = false;
+            }
+          }
+        }
+        if (exact) {
+          uint32_t pb[P];
+#pragma unroll
+          for (int x = 0; x < P; ++x) pb[x] = 0;
+          Tc = sim_exact<P, 1>(p, m, 1, F, B, C, br, pb, not_);
+          int len;
+          Mc = backtrack_master<P>(p, m, 1, br, pb, &len, NoEmit{});
+        }
+        s_chT[s][idx] = Tc;
+        s_chM[s][idx] = (int8_t)Mc;
+      }
+      atomicSub(&s_pend[s], 1);
+    }
+    __syncthreads();
+    if (tid == 0) s_head = head + nj;
+  }
+  if (A.stats) {
+    unsigned long long sm = my_sims, tr = my_trunc;
+#pragma unroll
+    for (int o = 16; o >= 1; o >>= 1) {
+      sm += __shfl_xor_sync(0xffffffffu, sm, o);
+      tr += __shfl_xor_sync(0xffffffffu, tr, o);
+    }
+    if ((tid & 31) == 0) {
+      if (sm) atomicAdd(&A.stats[0], sm);
+      if (tr) atomicAdd(&A.stats[1], tr);
+    }
+  }
+  block_min_atomic(my_key, A.key);
+}
 
 template <int P>
 __global__ void k_cpath(CpathArgs A) {
@@ -2430,9 +2698,47 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
   }
 }
 
+// Pool form of the reachable-set search (k_reach_pool, P <= 16, not the single-restart
+// decode replay); AP_REACH_POOL=0 keeps k_reach.  *lists_out = per-restart lists the
+// launch uses (scratch: lists x vmax entries).
+template <int P>
+static cudaError_t reach_pool_P(ReachArgs* A, cudaStream_t s, int dev, uint64_t R, bool launch,
+                                int* lists_out) {
+  const size_t narg = (size_t)(A->t.n + 1) * (A->p + 1);
+  const int rows = A->m + min(A->p - 1, A->m);
+  const size_t base = ((tables_smem_bytes(A->t.npad, A->t.n) + 15) & ~size_t(15)) +
+                      ((narg + 7) & ~size_t(7)) * 2 + 32 * 4;
+  const size_t smem = base + (size_t)rows * 4 * RP_NT;
+  if (smem > 160 * 1024) return cudaErrorInvalidValue;
+  cudaError_t e = cudaFuncSetAttribute((const void*)k_reach_pool<P>,
+                                       cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_reach_pool<P>, RP_NT, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  uint64_t blocks = (uint64_t)num_sms(dev) * occ;
+  const uint64_t need = (R + RP_NS - 1) / RP_NS;
+  if (blocks > need) blocks = need;
+  if (blocks < 1) blocks = 1;
+  *lists_out = (int)blocks * RP_NS;
+  if (!launch) return cudaSuccess;
+  k_reach_pool<P><<<(unsigned)blocks, RP_NT, smem, s>>>(*A);
+  return cudaGetLastError();
+}
+
+static bool reach_use_pool(const ReachArgs* A) {
+  const char* v = getenv("AP_REACH_POOL");
+  return !A->replay && pick_P(A->p) <= 16 && A->m + min(A->p - 1, A->m) <= 128 &&
+         A->vmax <= 2048 && !(v && v[0] == '0');
+}
+
 template <int P>
 static cudaError_t reach_P(ReachArgs* A, cudaStream_t s, int dev, uint64_t R, bool launch,
                            int* blocks_out) {
+  if constexpr (P <= 16) {
+    if (reach_use_pool(A)) return reach_pool_P<P>(A, s, dev, R, launch, blocks_out);
+  }
   const int threads = 128;
   const int rows = A->m + min(A->p - 1, A->m);
   const size_t narg = (size_t)(A->t.n + 1) * (A->p + 1);
@@ -2450,7 +2756,7 @@ static cudaError_t reach_P(ReachArgs* A, cudaStream_t s, int dev, uint64_t R, bo
   const uint64_t need = (R * 4 + threads - 1) / threads;
   if (blocks > need) blocks = need;
   if (blocks < 1) blocks = 1;
-  *blocks_out = (int)blocks;
+  *blocks_out = (int)blocks * 32;  // one list per quad
   if (!launch) return cudaSuccess;
   k_reach<P><<<(unsigned)blocks, threads, smem, s>>>(*A);
   return cudaGetLastError();
@@ -2467,6 +2773,13 @@ static cudaError_t reach_dispatch(ReachArgs* A, cudaStream_t s, int dev, uint64_
   }
 }
 
+// pool dedupe table entries per list: a power of two >= 2 * vmax (load <= 1/2)
+static size_t reach_tab_size(int vmax) {
+  size_t t = 64;
+  while (t < 2 * (size_t)vmax) t <<= 1;
+  return t;
+}
+
 cudaError_t reach_scratch_bytes(const DevTables& t, int p, int m, uint32_t R, int vmax,
                                 size_t* bytes) {
   int dev = 0;
@@ -2475,12 +2788,20 @@ cudaError_t reach_scratch_bytes(const DevTables& t, int p, int m, uint32_t R, in
   A.t = t;
   A.p = p;
   A.m = m;
-  int blocks = 0;
-  cudaError_t e = reach_dispatch(&A, nullptr, dev, R, false, &blocks);
+  A.vmax = vmax;
+  // the larger of the two kernels' list counts (the decode replay uses k_reach)
+  int lists = 0, lists_q = 0;
+  cudaError_t e = reach_dispatch(&A, nullptr, dev, R, false, &lists);
   if (e != cudaSuccess) return e;
-  const size_t quads = (size_t)blocks * 32;
+  int32_t dummy = 0;
+  A.replay = &dummy;
+  e = reach_dispatch(&A, nullptr, dev, R, false, &lists_q);
+  if (e != cudaSuccess) return e;
+  const size_t nl = (size_t)(lists > lists_q ? lists : lists_q);
   const size_t P = (size_t)pick_P(p);
-  *bytes = quads * (size_t)vmax * (P * 2 + 8) + 256;
+  A.replay = nullptr;
+  const size_t tab = reach_use_pool(&A) ? (size_t)lists * reach_tab_size(vmax) * 4 : 0;
+  *bytes = nl * (size_t)vmax * (P * 2 + 8) + tab + 512;
   return cudaSuccess;
 }
 
@@ -2507,18 +2828,26 @@ cudaError_t launch_reach(const DevTables& t, int p, int m, uint64_t seed, int ra
   A.vmax = vmax;
   A.stats = stats;
   A.replay = replay;
-  int blocks = 0;
-  cudaError_t e = reach_dispatch(&A, s, dev, r_hi - r_lo, false, &blocks);
+  int lists = 0;
+  cudaError_t e = reach_dispatch(&A, s, dev, r_hi - r_lo, false, &lists);
   if (e != cudaSuccess) return e;
-  const size_t quads = (size_t)blocks * 32;
+  const size_t nl = (size_t)lists;
   const size_t P = (size_t)pick_P(p);
   unsigned char* b = reinterpret_cast<unsigned char*>(scratch);
   A.g_cuts = reinterpret_cast<int16_t*>(b);
-  b += quads * (size_t)vmax * P * 2;
+  b += nl * (size_t)vmax * P * 2;
   A.g_hash = reinterpret_cast<uint32_t*>(b);
-  b += quads * (size_t)vmax * 4;
+  b += nl * (size_t)vmax * 4;
   A.g_queue = reinterpret_cast<uint32_t*>(b);
-  return reach_dispatch(&A, s, dev, r_hi - r_lo, true, &blocks);
+  b += nl * (size_t)vmax * 4;
+  if (reach_use_pool(&A)) {
+    b = reinterpret_cast<unsigned char*>(((uintptr_t)b + 255) & ~(uintptr_t)255);
+    A.g_tab = reinterpret_cast<uint32_t*>(b);
+    A.tab_size = (int)reach_tab_size(vmax);
+    e = cudaMemsetAsync(A.g_tab, 0, nl * (size_t)A.tab_size * 4, s);
+    if (e != cudaSuccess) return e;
+  }
+  return reach_dispatch(&A, s, dev, r_hi - r_lo, true, &lists);
 }
 
 size_t cpath_scratch_bytes(int p, int m) {

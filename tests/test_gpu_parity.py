@@ -972,3 +972,24 @@ def test_reach_fast_and_exact_simulation(ap, oracle_mod, monkeypatch, mode):
         assert (key >> 20, key & 0xFFFFF, sims, trunc) == (o["T"], o["restart"], o["sims"], o["truncated"]), (mode, p)
         res = ap.ap_decode_reachable(plan, p, m, 0x5EED, 2, 1024, key)
         assert res["time_ns"] == o["T"] and res["cuts"] == [int(x) for x in o["cuts"]]
+
+
+@pytest.mark.parametrize("pool", ["1", "0"])
+def test_reach_pool_and_quad_kernels(ap, oracle_mod, monkeypatch, pool):
+    """Both reachable-set kernels -- the simulation pool (default) and the 4-lane-group
+    kernel (AP_REACH_POOL=0; also used for vmax > 2048 and the decode replay) -- give
+    the oracle's winner, simulation count and truncations, incl. vmax > 2048."""
+    monkeypatch.setenv("AP_REACH_POOL", pool)
+    rng = np.random.default_rng(71)
+    for trial in range(6):
+        n = int(rng.integers(8, 40))
+        f, b, a = synth.random_tables(700 + trial, n, ["b3f", "uniform", "equal"][trial % 3])
+        bw = synth.link_for(["b3f", "uniform", "equal"][trial % 3])
+        M = oracle_mod.Model(f, b, a, bw)
+        plan = _plan(ap, f, b, a, bw)
+        p = int(rng.choice([2, 3, 4, 8]))
+        m = int(rng.integers(1, 3 * p))
+        vmax = int(rng.choice([2, 16, 1024, 4096]))
+        key, sims, trunc = _reach(ap, plan, p, m, 0x5EED, 2, 0, 150, vmax)
+        o = M.reach(p, m, 0x5EED, 2, 0, 150, vmax=vmax)
+        assert (key >> 20, key & 0xFFFFF, sims, trunc) == (o["T"], o["restart"], o["sims"], o["truncated"]), (pool, trial)

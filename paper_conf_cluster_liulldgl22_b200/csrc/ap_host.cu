@@ -466,8 +466,27 @@ ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t
   int launches = 0;
   static const int32_t kDummy = 0;
   (void)kDummy;
+  // u32 fast path: clamping every CR rows at S with
+  // (CR + p + 2) * W_row <= 2^32-1-S cannot wrap (a segment, the conversion row and the
+  // p cool-down rows; from 0 the warm-up is shorter), so every candidate with T < S is
+  // exact and the rest are recomputed in int64.  AP_EVAL=int64 disables it,
+  // AP_EVAL_S=<v> lowers S (tests of the fallback).
+  const int eCR = 16;
+  const unsigned __int128 wrow = (unsigned __int128)(plan->sum_f + plan->sum_b) +
+                                 (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
+  const unsigned __int128 need = wrow * (unsigned __int128)(eCR + p + 2);
+  const unsigned __int128 lim32 = ((unsigned __int128)1 << 32) - 1;
+  uint32_t fastS = need < lim32 ? (uint32_t)(lim32 - need) : 0u;
+  const char* ev = getenv("AP_EVAL");
+  if (ev && strcmp(ev, "int64") == 0) fastS = 0;
+  const char* es = getenv("AP_EVAL_S");
+  if (es && fastS > 0) {
+    const unsigned long long v = strtoull(es, nullptr, 10);
+    if (v > 0 && v < fastS) fastS = (uint32_t)v;
+  }
+  const int div1 = (plan->sum_f < (1ll << 28) && plan->max_comm < (1ll << 28)) ? 1 : 0;
   AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? cuts : nullptr, p - 1, k, 1, 0, count,
-                           time_ns, master, S_(stream), &launches));
+                           time_ns, master, S_(stream), &launches, 1, 0, fastS, eCR, div1));
   return AP_OK;
 }
 

@@ -751,227 +751,6 @@ __global__ void k_init_key(unsigned long long* key) { *key = 0x7fffffffffffffffu
 
 // ===========================================================================
 // K2 eval.
-struct EvalArgs {
-  DevTables t;
-  int p, m;
-  const int32_t* cuts;
-  int cuts_stride;
-  const int32_t* kptr;
-  int k_const, k_iota;
-  int64_t count;
-  int64_t* time_ns;
-  int32_t* master;
-  uint32_t* gbits;  // global bit scratch when shared memory is too small (or null)
-  int s_const;      // sliced leading micro-batches (1 = micro-batch 0 only, the default)
-  int s_iota;       // 1: row i uses s = i (paper-form slice sweep), k = k_const
-};
-
-template <int P>
-AP_DEV_INLINE bool load_cuts(const int32_t* row, int p, int n, int (&c)[P + 1]) {
-  bool ok = true;
-#pragma unroll
-  for (int x = 0; x <= P; ++x) c[x] = n;
-  c[0] = 0;
-  int prev = 0;
-#pragma unroll
-  for (int x = 1; x <= P - 1; ++x) {
-    if (x <= p - 1) {
-      const int v = row[x - 1];
-      ok = ok && (v > prev) && (v <= n - 1);
-      c[x] = v;
-      prev = v;
-    }
-  }
-  return ok;
-}
-
-template <int P>
-__global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  size_t used;
-  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= A.count) return;
-  const int p = A.p, m = A.m, n = A.t.n;
-  int c[P + 1];
-  const bool okc = load_cuts<P>(A.cuts + (size_t)i * A.cuts_stride, p, n, c);
-  const int k = A.kptr ? A.kptr[i] : (A.k_iota ? (int)(i + 1) : A.k_const);
-  const int sl = A.s_iota ? (int)i : A.s_const;
-  if (!okc || k < 1 || k > kMaxK || sl < 0 || sl > A.m) {
-    A.time_ns[i] = -1;
-    if (A.master) A.master[i] = -1;
-    return;
-  }
-  int64_t F[P], B[P], C[P];
-  stage_costs<P>(T, p, c, F, B, C);
-  if (sl != 1) {  // paper Slicer form: T only
-    A.time_ns[i] = sim_sliced<P>(p, m, sl, k, F, B, C);
-    if (A.master) A.master[i] = -1;
-    return;
-  }
-  uint32_t pb[P];
-  TimesRef not_{nullptr, nullptr, nullptr};
-  if (A.master == nullptr) {
-    BitsRef nob{nullptr, 0};
-    A.time_ns[i] = sim_exact<P, 0>(p, m, k, F, B, C, nob, pb, not_);
-    return;
-  }
-  BitsRef br;
-  if (A.gbits) {
-    br.base = A.gbits + i;
-    br.stride = (int)A.count;
-  } else {
-    uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + ((used + 15) & ~size_t(15)));
-    br.base = sbits + threadIdx.x;
-    br.stride = blockDim.x;
-  }
-  A.time_ns[i] = sim_exact<P, 1>(p, m, k, F, B, C, br, pb, not_);
-  int len;
-  A.master[i] = backtrack_master<P>(p, m, k, br, pb, &len, NoEmit{});
-}
-
-// ===========================================================================
-// Algorithm 1 (PAPER.md:158-188), one CTA.  time[0][0] = 0, others +inf;
-// time[i][j] = min_k max(time[k][j-1], P[i]-P[k]) over k ascending, strict '<'
-// (smallest k wins ties); the arg table drives line 15's reconstruction.
-__global__ void __launch_bounds__(256) k_alg1(DevTables t, int p, int16_t* arg, int32_t* cuts,
-                                              int64_t* value) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  size_t used;
-  const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
-  const int n = t.n, P1 = p + 1;
-  int64_t* tt = reinterpret_cast<int64_t*>(smem + ((used + 15) & ~size_t(15)));
-  // prefix_sum of f+b (line 6): Pf + Pb
-  for (int e = threadIdx.x; e < (n + 1) * P1; e += blockDim.x) {
-    tt[e] = (e == 0) ? 0 : INT64_MAX;
-    arg[e] = -1;
-  }
-  __syncthreads();
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-  for (int i = 1; i <= n; ++i) {
-    const int64_t Pi = T.Pf[i] + T.Pb[i];
-    const int jmax = min(p, i);
-    for (int j = 1 + warp; j <= jmax; j += nw) {
-      int64_t bv = INT64_MAX;
-      int bk = INT32_MAX;
-      for (int kk = lane; kk <= i - 1; kk += 32) {
-        const int64_t prev = tt[kk * P1 + (j - 1)];
-        const int64_t seg = Pi - (T.Pf[kk] + T.Pb[kk]);
-        const int64_t v = prev > seg ? prev : seg;
-        if (v < bv) {  // kk ascending within the lane: first wins
-          bv = v;
-          bk = kk;
-        }
-      }
-#pragma unroll
-      for (int o = 16; o >= 1; o >>= 1) {
-        const int64_t ov = __shfl_xor_sync(0xffffffffu, bv, o);
-        const int ok = __shfl_xor_sync(0xffffffffu, bk, o);
-        if (ov < bv || (ov == bv && ok < bk)) {
-          bv = ov;
-          bk = ok;
-        }
-      }
-      if (lane == 0 && bv != INT64_MAX) {
-        tt[i * P1 + j] = bv;
-        arg[i * P1 + j] = (int16_t)bk;
-      }
-    }
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    *value = tt[n * P1 + p];
-    int e = n;
-    for (int jj = p; jj >= 2; --jj) {
-      const int st = arg[e * P1 + jj];
-      cuts[jj - 2] = st;
-      e = st;
-    }
-  }
-}
-
-// ===========================================================================
-// Certified minLB (SURVEY P14, NEXT N3; DESIGN.md reading R-LB), one CTA.  Per-stage
-// relaxation of the O11 bound, g(x, a, b) for stage x = [a, b):
-//   ceil+((Pf[a] - x(K-1)) / K) + (x-1) floor(cmin/K)              (fill)
-//   + m (F + B + [x>0] comm[a-1] + [x<p-1] comm[b-1])              (busy)
-//   + Pb[a] + [x>0] (comm[a-1] + (x-1) cmin)                       (tail)
-// bottleneck DP D[x+1][b] = min_a max(D[x][a], g), a ascending, strict '<'.
-AP_DEV_INLINE int64_t minlb_term(const Tables& T, int p, int m, int K, int64_t cmin, int x,
-                                 int a, int b) {
-  int64_t fill = T.Pf[a] - (int64_t)x * (K - 1);
-  fill = fill <= 0 ? 0 : (fill + K - 1) / K;
-  const int64_t cin = x > 0 ? T.comm[a - 1] : 0;
-  const int64_t cout = x < p - 1 ? T.comm[b - 1] : 0;
-  if (x > 0) fill += (int64_t)(x - 1) * (cmin / K);
-  const int64_t busy = (int64_t)m * (T.Pf[b] - T.Pf[a] + T.Pb[b] - T.Pb[a] + cin + cout);
-  const int64_t tail = T.Pb[a] + (x > 0 ? cin + (int64_t)(x - 1) * cmin : 0);
-  return fill + busy + tail;
-}
-
-__global__ void __launch_bounds__(256) k_minlb(DevTables t, int p, int m, int K, int16_t* arg,
-                                               int32_t* cuts, int64_t* value) {
-  extern __shared__ __align__(16) unsigned char smem[];
-  size_t used;
-  const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
-  const int n = t.n, N1 = n + 1;
-  int64_t* D = reinterpret_cast<int64_t*>(smem + ((used + 15) & ~size_t(15)));
-  __shared__ int64_t s_cmin;
-  for (int e = threadIdx.x; e < (p + 1) * N1; e += blockDim.x) {
-    D[e] = (e == 0) ? 0 : INT64_MAX;
-    arg[e] = -1;
-  }
-  if (threadIdx.x == 0) {
-    int64_t c = 0;
-    for (int i = 0; i + 1 < n; ++i) c = (i == 0 || T.comm[i] < c) ? T.comm[i] : c;
-    s_cmin = c;
-  }
-  __syncthreads();
-  const int64_t cmin = s_cmin;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-  for (int x = 0; x < p; ++x) {
-    const int b_lo = (x == p - 1) ? n : x + 1, b_hi = n - (p - 1 - x);
-    for (int b = b_lo + warp; b <= b_hi; b += nw) {
-      int64_t bv = INT64_MAX;
-      int ba = INT32_MAX;
-      for (int a = x + lane; a < b; a += 32) {
-        const int64_t prev = D[x * N1 + a];
-        if (prev == INT64_MAX) continue;
-        const int64_t g = minlb_term(T, p, m, K, cmin, x, a, b);
-        const int64_t v = prev > g ? prev : g;
-        if (v < bv) {  // a ascending within the lane: first wins
-          bv = v;
-          ba = a;
-        }
-      }
-#pragma unroll
-      for (int o = 16; o >= 1; o >>= 1) {
-        const int64_t ov = __shfl_xor_sync(0xffffffffu, bv, o);
-        const int oa = __shfl_xor_sync(0xffffffffu, ba, o);
-        if (ov < bv || (ov == bv && oa < ba)) {
-          bv = ov;
-          ba = oa;
-        }
-      }
-      if (lane == 0 && bv != INT64_MAX) {
-        D[(x + 1) * N1 + b] = bv;
-        arg[(x + 1) * N1 + b] = (int16_t)ba;
-      }
-    }
-    __syncthreads();
-  }
-  if (threadIdx.x == 0) {
-    *value = D[p * N1 + n];
-    int e = n;
-    for (int x = p; x >= 2; --x) {
-      e = arg[x * N1 + e];
-      cuts[x - 2] = e;
-    }
-  }
-}
-
-// ===========================================================================
-// K3 heuristic restarts (adjust_mode none; reading O9).
 // u32 saturating p-specialised simulation (k = 1, p == P, m >= P) that also writes
 // the decision bits the backtrack reads, in exactly the layout of sim_exact (rows
 // y + W0 = r; F bit x, B bit 16+x).  It is the M-form sweep of sweep_tail: B(x, y) and
@@ -1125,6 +904,297 @@ AP_DEV_INLINE int backtrack_master_bl(int m, BitsRef br) {
   return best;
 }
 
+struct EvalArgs {
+  DevTables t;
+  int p, m;
+  const int32_t* cuts;
+  int cuts_stride;
+  const int32_t* kptr;
+  int k_const, k_iota;
+  int64_t count;
+  int64_t* time_ns;
+  int32_t* master;
+  uint32_t* gbits;  // global bit scratch when shared memory is too small (or null)
+  int s_const;      // sliced leading micro-batches (1 = micro-batch 0 only, the default)
+  int s_iota;       // 1: row i uses s = i (paper-form slice sweep), k = k_const
+  uint32_t fastS;   // > 0: u32 fast path (p == P <= 16, m >= P, s = 1) exact below fastS,
+                    // clamped every CR rows; a result >= fastS is recomputed in int64
+  int CR, div1;     // clamp interval; one-umulhi pieces (see divk)
+  // fast pass: a candidate whose u32 result reaches fastS is appended to redo (count at
+  // redo[0], indices at redo[1..]) instead of diverging its warp into the int64 path;
+  // redo pass (fastS = 0, redo_in set): evaluates exactly the listed candidates
+  unsigned int* redo;
+  const unsigned int* redo_in;
+};
+// u32 copies of the prefix sums / comm and the floor(v/k) magics for the fast path
+__host__ __device__ inline size_t eval_fast_smem(int n) {
+  return ((size_t)(2 * n + 1 + kMaxK + 1) * 4 + 15) & ~size_t(15);
+}
+
+template <int P>
+AP_DEV_INLINE bool load_cuts(const int32_t* row, int p, int n, int (&c)[P + 1]) {
+  bool ok = true;
+#pragma unroll
+  for (int x = 0; x <= P; ++x) c[x] = n;
+  c[0] = 0;
+  int prev = 0;
+#pragma unroll
+  for (int x = 1; x <= P - 1; ++x) {
+    if (x <= p - 1) {
+      const int v = row[x - 1];
+      ok = ok && (v > prev) && (v <= n - 1);
+      c[x] = v;
+      prev = v;
+    }
+  }
+  return ok;
+}
+
+template <int P>
+__global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  size_t off = (used + 15) & ~size_t(15);
+  uint32_t *s32Pf = nullptr, *s32C = nullptr, *s32mk = nullptr;
+  if (A.fastS) {  // block-uniform
+    s32Pf = reinterpret_cast<uint32_t*>(smem + off);
+    s32C = s32Pf + (A.t.n + 1);
+    s32mk = s32C + A.t.n;
+    for (int e = threadIdx.x; e <= A.t.n; e += blockDim.x) {
+      s32Pf[e] = (uint32_t)T.Pf[e];
+      if (e < A.t.n) s32C[e] = (uint32_t)T.comm[e];
+    }
+    if (threadIdx.x <= kMaxK)
+      s32mk[threadIdx.x] = (threadIdx.x <= 1) ? 0xffffffffu
+                           : A.div1 ? (uint32_t)(((1ull << 32) + threadIdx.x - 1) / threadIdx.x)
+                                    : (uint32_t)((1ull << 32) / threadIdx.x);
+    off += eval_fast_smem(A.t.n);
+    __syncthreads();
+  }
+  const int p = A.p, m = A.m, n = A.t.n;
+  // grid-stride (persistent) loop: the table prologue above runs once per CTA
+  const int64_t cnt = A.redo_in ? (int64_t)A.redo_in[0] : A.count;
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < cnt;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = A.redo_in ? (int64_t)A.redo_in[1 + j] : j;
+
+    int c[P + 1];
+    const bool okc = load_cuts<P>(A.cuts + (size_t)i * A.cuts_stride, p, n, c);
+    const int k = A.kptr ? A.kptr[i] : (A.k_iota ? (int)(i + 1) : A.k_const);
+    const int sl = A.s_iota ? (int)i : A.s_const;
+    if (!okc || k < 1 || k > kMaxK || sl < 0 || sl > A.m) {
+      A.time_ns[i] = -1;
+      if (A.master) A.master[i] = -1;
+      continue;
+    }
+    int64_t F[P], B[P], C[P];
+    stage_costs<P>(T, p, c, F, B, C);
+    if (sl != 1) {  // paper Slicer form: T only
+      A.time_ns[i] = sim_sliced<P>(p, m, sl, k, F, B, C);
+      if (A.master) A.master[i] = -1;
+      continue;
+    }
+    uint32_t pb[P];
+    TimesRef not_{nullptr, nullptr, nullptr};
+    BitsRef br{nullptr, 0};
+    if (A.master) {
+      if (A.gbits) {
+        br.base = A.gbits + i;
+        br.stride = (int)A.count;
+      } else {
+        uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + off);
+        br.base = sbits + threadIdx.x;
+        br.stride = blockDim.x;
+      }
+    }
+    if constexpr (P >= 2 && P <= 16) {
+      // u32 fast path: the N-form sweep (T only) or the M-form with decision bits and
+      // the branch-free backtrack (k = 1); exact below fastS
+      if (A.fastS && p == P && m >= P && m <= 32767) {
+        uint32_t wF[P], wB[P];
+  #pragma unroll
+        for (int x = 0; x < P; ++x) {
+          wF[x] = (uint32_t)(F[x] + ((x > 0) ? C[x - 1] : 0));
+          wB[x] = (uint32_t)(B[x] + C[x]);
+        }
+        if (A.master == nullptr) {
+          const ClampSched cs{0, A.CR, 1};
+          const uint32_t t32 = sim_fast<P, uint32_t>(m, k, wF, wB, c, s32Pf, s32C, s32mk[k],
+                                                     A.div1 != 0, A.fastS, cs, 1u);
+          if (t32 < A.fastS) {
+            A.time_ns[i] = (int64_t)t32;
+          } else {
+            A.redo[1 + atomicAdd(&A.redo[0], 1u)] = (unsigned int)i;
+          }
+          continue;
+        } else if (k == 1) {
+          const uint32_t t32 = sim_fast_bits<P>(m, wF, wB, A.fastS, A.CR, br);
+          if (t32 < A.fastS) {
+            A.time_ns[i] = (int64_t)t32;
+            A.master[i] = m <= 127 ? backtrack_master_bl<P, 8>(m, br) : backtrack_master_bl<P, 16>(m, br);
+          } else {
+            A.redo[1 + atomicAdd(&A.redo[0], 1u)] = (unsigned int)i;
+          }
+          continue;
+        }
+      }
+    }
+    if (A.master == nullptr) {
+      BitsRef nob{nullptr, 0};
+      A.time_ns[i] = sim_exact<P, 0>(p, m, k, F, B, C, nob, pb, not_);
+      continue;
+    }
+    A.time_ns[i] = sim_exact<P, 1>(p, m, k, F, B, C, br, pb, not_);
+    int len;
+    A.master[i] = backtrack_master<P>(p, m, k, br, pb, &len, NoEmit{});
+  }
+}
+
+// ===========================================================================
+// Algorithm 1 (PAPER.md:158-188), one CTA.  time[0][0] = 0, others +inf;
+// time[i][j] = min_k max(time[k][j-1], P[i]-P[k]) over k ascending, strict '<'
+// (smallest k wins ties); the arg table drives line 15's reconstruction.
+__global__ void __launch_bounds__(256) k_alg1(DevTables t, int p, int16_t* arg, int32_t* cuts,
+                                              int64_t* value) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
+  const int n = t.n, P1 = p + 1;
+  int64_t* tt = reinterpret_cast<int64_t*>(smem + ((used + 15) & ~size_t(15)));
+  // prefix_sum of f+b (line 6): Pf + Pb
+  for (int e = threadIdx.x; e < (n + 1) * P1; e += blockDim.x) {
+    tt[e] = (e == 0) ? 0 : INT64_MAX;
+    arg[e] = -1;
+  }
+  __syncthreads();
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int i = 1; i <= n; ++i) {
+    const int64_t Pi = T.Pf[i] + T.Pb[i];
+    const int jmax = min(p, i);
+    for (int j = 1 + warp; j <= jmax; j += nw) {
+      int64_t bv = INT64_MAX;
+      int bk = INT32_MAX;
+      for (int kk = lane; kk <= i - 1; kk += 32) {
+        const int64_t prev = tt[kk * P1 + (j - 1)];
+        const int64_t seg = Pi - (T.Pf[kk] + T.Pb[kk]);
+        const int64_t v = prev > seg ? prev : seg;
+        if (v < bv) {  // kk ascending within the lane: first wins
+          bv = v;
+          bk = kk;
+        }
+      }
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) {
+        const int64_t ov = __shfl_xor_sync(0xffffffffu, bv, o);
+        const int ok = __shfl_xor_sync(0xffffffffu, bk, o);
+        if (ov < bv || (ov == bv && ok < bk)) {
+          bv = ov;
+          bk = ok;
+        }
+      }
+      if (lane == 0 && bv != INT64_MAX) {
+        tt[i * P1 + j] = bv;
+        arg[i * P1 + j] = (int16_t)bk;
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    *value = tt[n * P1 + p];
+    int e = n;
+    for (int jj = p; jj >= 2; --jj) {
+      const int st = arg[e * P1 + jj];
+      cuts[jj - 2] = st;
+      e = st;
+    }
+  }
+}
+
+// ===========================================================================
+// Certified minLB (SURVEY P14, NEXT N3; DESIGN.md reading R-LB), one CTA.  Per-stage
+// relaxation of the O11 bound, g(x, a, b) for stage x = [a, b):
+//   ceil+((Pf[a] - x(K-1)) / K) + (x-1) floor(cmin/K)              (fill)
+//   + m (F + B + [x>0] comm[a-1] + [x<p-1] comm[b-1])              (busy)
+//   + Pb[a] + [x>0] (comm[a-1] + (x-1) cmin)                       (tail)
+// bottleneck DP D[x+1][b] = min_a max(D[x][a], g), a ascending, strict '<'.
+AP_DEV_INLINE int64_t minlb_term(const Tables& T, int p, int m, int K, int64_t cmin, int x,
+                                 int a, int b) {
+  int64_t fill = T.Pf[a] - (int64_t)x * (K - 1);
+  fill = fill <= 0 ? 0 : (fill + K - 1) / K;
+  const int64_t cin = x > 0 ? T.comm[a - 1] : 0;
+  const int64_t cout = x < p - 1 ? T.comm[b - 1] : 0;
+  if (x > 0) fill += (int64_t)(x - 1) * (cmin / K);
+  const int64_t busy = (int64_t)m * (T.Pf[b] - T.Pf[a] + T.Pb[b] - T.Pb[a] + cin + cout);
+  const int64_t tail = T.Pb[a] + (x > 0 ? cin + (int64_t)(x - 1) * cmin : 0);
+  return fill + busy + tail;
+}
+
+__global__ void __launch_bounds__(256) k_minlb(DevTables t, int p, int m, int K, int16_t* arg,
+                                               int32_t* cuts, int64_t* value) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
+  const int n = t.n, N1 = n + 1;
+  int64_t* D = reinterpret_cast<int64_t*>(smem + ((used + 15) & ~size_t(15)));
+  __shared__ int64_t s_cmin;
+  for (int e = threadIdx.x; e < (p + 1) * N1; e += blockDim.x) {
+    D[e] = (e == 0) ? 0 : INT64_MAX;
+    arg[e] = -1;
+  }
+  if (threadIdx.x == 0) {
+    int64_t c = 0;
+    for (int i = 0; i + 1 < n; ++i) c = (i == 0 || T.comm[i] < c) ? T.comm[i] : c;
+    s_cmin = c;
+  }
+  __syncthreads();
+  const int64_t cmin = s_cmin;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
+  for (int x = 0; x < p; ++x) {
+    const int b_lo = (x == p - 1) ? n : x + 1, b_hi = n - (p - 1 - x);
+    for (int b = b_lo + warp; b <= b_hi; b += nw) {
+      int64_t bv = INT64_MAX;
+      int ba = INT32_MAX;
+      for (int a = x + lane; a < b; a += 32) {
+        const int64_t prev = D[x * N1 + a];
+        if (prev == INT64_MAX) continue;
+        const int64_t g = minlb_term(T, p, m, K, cmin, x, a, b);
+        const int64_t v = prev > g ? prev : g;
+        if (v < bv) {  // a ascending within the lane: first wins
+          bv = v;
+          ba = a;
+        }
+      }
+#pragma unroll
+      for (int o = 16; o >= 1; o >>= 1) {
+        const int64_t ov = __shfl_xor_sync(0xffffffffu, bv, o);
+        const int oa = __shfl_xor_sync(0xffffffffu, ba, o);
+        if (ov < bv || (ov == bv && oa < ba)) {
+          bv = ov;
+          ba = oa;
+        }
+      }
+      if (lane == 0 && bv != INT64_MAX) {
+        D[(x + 1) * N1 + b] = bv;
+        arg[(x + 1) * N1 + b] = (int16_t)ba;
+      }
+    }
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) {
+    *value = D[p * N1 + n];
+    int e = n;
+    for (int x = p; x >= 2; --x) {
+      e = arg[x * N1 + e];
+      cuts[x - 2] = e;
+    }
+  }
+}
+
+// ===========================================================================
+// K3 heuristic restarts (adjust_mode none; reading O9).  The u32
+// simulation with decision bits (sim_fast_bits) and the branch-free master backtrack
+// (backtrack_master_bl) are defined above, next to K2, which shares them.
 struct HeurArgs {
   DevTables t;
   int p, m;
@@ -2398,7 +2468,8 @@ cudaError_t launch_minlb(const DevTables& t, int p, int m, int K, int16_t* arg, 
 template <int P>
 static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   EvalArgs A = A0;
-  const size_t base = (tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15);
+  const size_t base = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
+                      (A.fastS ? eval_fast_smem(A.t.n) : 0);
   int threads = 128;
   size_t smem = base;
   if (A.master) {
@@ -2416,7 +2487,15 @@ static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   }
   cudaError_t e = set_smem((const void*)k_eval<P>, smem);
   if (e != cudaSuccess) return e;
-  const int64_t blocks = (A.count + threads - 1) / threads;
+  // persistent grid: at most one wave (the kernel strides over the candidates)
+  int occ = 0, dev = 0;
+  cudaGetDevice(&dev);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval<P>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  int64_t blocks = (A.count + threads - 1) / threads;
+  const int64_t wave = (int64_t)num_sms(dev) * occ;
+  if (blocks > wave) blocks = wave;  // (redo pass: the listed count is <= A.count)
   if (blocks > 0) {
     k_eval<P><<<(unsigned)blocks, threads, smem, s>>>(A);
     if (launches) ++*launches;
@@ -2428,15 +2507,25 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
                         int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
                         int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches,
-                        int s_const, int s_iota) {
+                        int s_const, int s_iota, uint32_t fastS, int fastCR, int div1) {
   EvalArgs A{t, p, m, cuts, cuts_stride, kptr, k_const, k_iota, count, time_ns, master, nullptr,
-             s_const, s_iota};
+             s_const, s_iota, fastS, fastCR < 1 ? 1 : fastCR, div1, nullptr, nullptr};
   uint32_t* gbits = nullptr;
+  unsigned int* redo = nullptr;
+  if (fastS && count >= (1ll << 32)) fastS = A.fastS = 0;  // redo indices are 32-bit
+  if (fastS) {
+    cudaError_t e = cudaMallocFromPoolAsync((void**)&redo, 4 * ((size_t)count + 1), pool, s);
+    if (e != cudaSuccess) return e;
+    e = cudaMemsetAsync(redo, 0, 4, s);
+    if (e != cudaSuccess) return e;
+    A.redo = redo;
+  }
   if (master) {
     const int rows = m + min(p - 1, m);
     const int P = pick_P(p);
     const size_t per = (size_t)rows * (P <= 16 ? 1 : 2) * 4;
-    const size_t base = (tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15);
+    const size_t base = ((tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15)) +
+                        (fastS ? eval_fast_smem(t.n) : 0);
     if (per * 32 > 200 * 1024 - base) {
       cudaError_t e = cudaMallocFromPoolAsync((void**)&gbits, per * (size_t)count + 16, pool, s);
       if (e != cudaSuccess) return e;
@@ -2444,14 +2533,27 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
     }
   }
   cudaError_t e;
-  switch (pick_P(p)) {
-    case 2: e = eval_P<2>(A, s, launches); break;
-    case 4: e = eval_P<4>(A, s, launches); break;
-    case 8: e = eval_P<8>(A, s, launches); break;
-    case 16: e = eval_P<16>(A, s, launches); break;
-    default: e = eval_P<32>(A, s, launches); break;
+  auto run = [&](const EvalArgs& X) {
+    switch (pick_P(p)) {
+      case 2: return eval_P<2>(X, s, launches);
+      case 4: return eval_P<4>(X, s, launches);
+      case 8: return eval_P<8>(X, s, launches);
+      case 16: return eval_P<16>(X, s, launches);
+      default: return eval_P<32>(X, s, launches);
+    }
+  };
+  e = run(A);
+  if (e == cudaSuccess && redo) {
+    // exact int64 pass over the candidates that reached the u32 bound (one wave; it
+    // reads the count on the device and exits at once when the list is empty)
+    EvalArgs X = A;
+    X.fastS = 0;
+    X.redo = nullptr;
+    X.redo_in = redo;
+    e = run(X);
   }
   if (gbits) cudaFreeAsync(gbits, s);
+  if (redo) cudaFreeAsync(redo, s);
   return e;
 }
 

@@ -29,7 +29,8 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
                         int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
                         int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches,
-                        int s_const = 1, int s_iota = 0);
+                        int s_const = 1, int s_iota = 0, uint32_t fastS = 0, int fastCR = 16,
+                        int div1 = 0);
 
 struct SweepPlan {
   int fast_u32;   // exact u32 saturating sweep

@@ -993,3 +993,41 @@ def test_reach_pool_and_quad_kernels(ap, oracle_mod, monkeypatch, pool):
         key, sims, trunc = _reach(ap, plan, p, m, 0x5EED, 2, 0, 150, vmax)
         o = M.reach(p, m, 0x5EED, 2, 0, 150, vmax=vmax)
         assert (key >> 20, key & 0xFFFFF, sims, trunc) == (o["T"], o["restart"], o["sims"], o["truncated"]), (pool, trial)
+
+
+@pytest.mark.parametrize("mode", ["fast", "int64", "saturating"])
+def test_eval_batch_fast_path(ap, oracle_mod, monkeypatch, mode):
+    """ap_eval_batch's u32 fast path (p in {2,4,8,16}, m >= p: N-form sweep for T, the
+    bit-recording sweep + branch-free backtrack for T + master at k = 1), the exact
+    int64 kernel (AP_EVAL=int64) and the fast path with a bound low enough that many
+    candidates fall back to int64 (AP_EVAL_S): T and master equal the oracle's for
+    every candidate, k up to 16."""
+    import torch
+    if mode == "int64":
+        monkeypatch.setenv("AP_EVAL", "int64")
+    rng = np.random.default_rng(83)
+    for trial, p in enumerate((2, 4, 8, 16, 8)):
+        n = int(rng.integers(p + 2, 3 * p + 20))
+        kind = ["b3f", "uniform", "equal", "small", "huge"][trial]
+        f, b, a = synth.random_tables(1200 + trial, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        m = int(rng.integers(p, 3 * p + 3))
+        cnt = 64
+        cuts = np.sort(np.argsort(rng.random((cnt, n - 1)), axis=1)[:, : p - 1] + 1, axis=1).astype(np.int32)
+        ks = rng.integers(1, 17, cnt).astype(np.int32)
+        want = [M.simulate(p, m, list(c), k=int(k))["T"] for c, k in zip(cuts, ks)]
+        if mode == "saturating":
+            monkeypatch.setenv("AP_EVAL_S", str(int(np.median(want))))
+        plan = _plan(ap, f, b, a, bw)
+        dc = torch.from_numpy(cuts).cuda()
+        T = torch.empty(cnt, dtype=torch.int64, device="cuda")
+        ap.ap_eval_batch(plan, p, m, dc, torch.from_numpy(ks).cuda(), T)
+        torch.cuda.synchronize()
+        assert T.tolist() == want, (mode, p, kind)
+        k1 = torch.ones(cnt, dtype=torch.int32, device="cuda")
+        Mst = torch.empty(cnt, dtype=torch.int32, device="cuda")
+        ap.ap_eval_batch(plan, p, m, dc, k1, T, Mst)
+        torch.cuda.synchronize()
+        o = [M.simulate(p, m, list(c)) for c in cuts]
+        assert T.tolist() == [x["T"] for x in o] and Mst.tolist() == [x["master"] for x in o], (mode, p, kind)

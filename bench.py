@@ -551,6 +551,37 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
                        "sims_per_step": sum(r["sims"] for r in r4["per_depth"]),
                        "best": {k: r4["best"][k] for k in ("p", "dp", "m", "T", "cuts")},
                        "per_depth_T_ns": {r["p"]: r["T"] for r in r4["per_depth"]}}
+
+    # ap_eval_batch on 2^24 random C4 candidates per rank (T with k in 1..8; T + master
+    # at k = 1): the general evaluation entry point, candidates resident in HBM
+    wl = synth.config(4)
+    f, b, a = wl.arrays()
+    plan5 = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=dev.index)
+    cnt = 1 << 24
+    g = torch.Generator(device=dev)
+    g.manual_seed(1234 + rank)
+    cuts = torch.sort(torch.argsort(torch.rand(cnt, wl.n - 1, device=dev, generator=g), dim=1)
+                      [:, : wl.p - 1] + 1, dim=1).values.to(torch.int32).contiguous()
+    ks = torch.randint(wl.k_lo, wl.k_hi + 1, (cnt,), device=dev, generator=g, dtype=torch.int32)
+    k1 = torch.ones(cnt, dtype=torch.int32, device=dev)
+    Tv = torch.empty(cnt, dtype=torch.int64, device=dev)
+    Mv = torch.empty(cnt, dtype=torch.int32, device=dev)
+    ev = {}
+    for name, kk, mm in (("T", ks, None), ("T_master_k1", k1, Mv)):
+        ap.ap_eval_batch(plan5, wl.p, wl.m, cuts, kk, Tv, mm)
+        times = []
+        for _ in range(5):
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(); ap.ap_eval_batch(plan5, wl.p, wl.m, cuts, kk, Tv, mm); e1.record()
+            torch.cuda.synchronize()
+            times.append(e0.elapsed_time(e1))
+        t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ev[name] = {"ms": float(t[0]), "sims_per_s": world * cnt / (float(t[0]) / 1e3)}
+    del cuts, ks, k1, Tv, Mv
+    out["eval_batch"] = {"workload": "C4 random partitions, 2^24 per rank", **ev}
     return out
 
 

@@ -552,12 +552,12 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
                        "best": {k: r4["best"][k] for k in ("p", "dp", "m", "T", "cuts")},
                        "per_depth_T_ns": {r["p"]: r["T"] for r in r4["per_depth"]}}
 
-    # ap_eval_batch on 2^24 random C4 candidates per rank (T with k in 1..8; T + master
+    # ap_eval_batch on 2^22 random C4 candidates per rank (T with k in 1..8; T + master
     # at k = 1): the general evaluation entry point, candidates resident in HBM
     wl = synth.config(4)
     f, b, a = wl.arrays()
     plan5 = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=dev.index)
-    cnt = 1 << 24
+    cnt = 1 << 22
     g = torch.Generator(device=dev)
     g.manual_seed(1234 + rank)
     cuts = torch.sort(torch.argsort(torch.rand(cnt, wl.n - 1, device=dev, generator=g), dim=1)
@@ -581,7 +581,7 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
         ev[name] = {"ms": float(t[0]), "sims_per_s": world * cnt / (float(t[0]) / 1e3)}
     del cuts, ks, k1, Tv, Mv
-    out["eval_batch"] = {"workload": "C4 random partitions, 2^24 per rank", **ev}
+    out["eval_batch"] = {"workload": "C4 random partitions, 2^22 per rank", **ev}
     return out
 
 

@@ -792,6 +792,79 @@ AP_DEV_INLINE uint32_t sim_fast_bits(int m, const uint32_t (&wF)[P], const uint3
   for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
   int r = P - 1;
   int rem = m - P;
+#if AP_NFORM
+  if constexpr (P >= 3) {
+    // offset form with the same decision bits: the first step in the
+    // M-form below keeps N = M - c; then per stage t = N'[x+1] + s[x+1],
+    // gt_x = N[x-1] > t (i.e. FF[x] > b[x+1]), N'[x] = max(t, N[x-1]), and at x = 0 the
+    // intra operand is N[0] + s[0].  Clamps apply to N; the conversion back sits at
+    // most one row's growth above S, inside heur_fast_bound's margin.
+    if (rem > 0) {
+      uint32_t c[P], sw[P], N[P];
+      c[0] = wF[0];
+#pragma unroll
+      for (int x = 1; x < P; ++x) c[x] = c[x - 1] + wF[x];
+#pragma unroll
+      for (int x = 0; x < P; ++x) sw[x] = wF[x] + wB[x];
+      {  // first step, M-form
+        uint32_t wordF = 0;
+        uint32_t b = FF[P - 1] + wB[P - 1];
+#pragma unroll
+        for (int x = P - 2; x >= 0; --x) {
+          const bool gt = FF[x] > b;
+          if (gt) wordF |= 1u << (x + 1);
+          const uint32_t M = max(FF[x], b);
+          N[x] = M - c[x];
+          b = M + wB[x];
+        }
+        const uint32_t wordB = ((~wordF >> 1) & ((1u << (P - 1)) - 1u)) << 16;
+        br.base[(size_t)r * br.stride] = nxt | wordB;
+        nxt = wordF;
+        ++r;
+      }
+      int blk = (rem < CR ? rem : CR) - 1;
+      rem -= blk + 1;
+      for (;;) {
+        for (; blk > 0; --blk) {
+          uint32_t wordF = 0, n[P];
+          uint32_t t = N[P - 2] + sw[P - 1];
+          bool gt = N[P - 3 >= 0 ? P - 3 : 0] > t;
+          if (P >= 3) {
+            if (gt) wordF |= 1u << (P - 1);
+            n[P - 2] = max(N[P - 3], t);
+          }
+#pragma unroll
+          for (int x = P - 3; x >= 1; --x) {
+            t = n[x + 1] + sw[x + 1];
+            gt = N[x - 1] > t;
+            if (gt) wordF |= 1u << (x + 1);
+            n[x] = max(N[x - 1], t);
+          }
+          t = n[1] + sw[1];
+          const uint32_t u = N[0] + sw[0];
+          gt = u > t;
+          if (gt) wordF |= 1u << 1;
+          n[0] = max(u, t);
+#pragma unroll
+          for (int x = 0; x <= P - 2; ++x) N[x] = n[x];
+          const uint32_t wordB = ((~wordF >> 1) & ((1u << (P - 1)) - 1u)) << 16;
+          br.base[(size_t)r * br.stride] = nxt | wordB;
+          nxt = wordF;
+          ++r;
+        }
+#pragma unroll
+        for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
+        if (rem <= 0) break;
+        blk = rem < CR ? rem : CR;
+        rem -= blk;
+      }
+#pragma unroll
+      for (int x = 0; x <= P - 2; ++x) FF[x + 1] = N[x] + c[x + 1];
+      FF[0] = N[0] + c[0] + sw[0];
+    }
+    rem = 0;
+  }
+#endif
   while (rem > 0) {
     int blk = rem < CR ? rem : CR;
     rem -= blk;

@@ -1562,9 +1562,8 @@ constexpr int RING = 512; // job ring, >= 4 * NS
 }  // namespace hpool
 
 // Child idx (0 a, 1 a', 2 b, 3 b') of `cur` with master i (
-// reading Q17), as k_heur's gen_child; false if invalid or a duplicate.
 // reading Q17), as k_heur's gen_child, built in place in shared memory (no local
-// arrays); false if invalid or a duplicate.
+// arrays); false if invalid or a duplicate (a' == a, b' == b).
 AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
                               const int16_t* s_arg, int16_t* cand) {
   if (cur[i + 1] - cur[i] < 2) return false;

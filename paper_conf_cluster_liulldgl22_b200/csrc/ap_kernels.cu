@@ -589,17 +589,41 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
         // cannot hold a candidate with T < S = T_ref + 1.
         // (64-bit: m * load can exceed 2^32 for the heavy partitions it prunes)
         const uint32_t Kh = (uint32_t)k_hi, MK = s_mk[k_hi];
-        uint64_t fill = 0, tail = 0, lb = 0;
+        uint64_t fill = 0, tail = 0;
+        int xf = P;  // first stage whose bound reaches S
 #pragma unroll
         for (int x = 0; x < P; ++x) {
           const V Fx = sPf[c[x + 1]] - sPf[c[x]];
           const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
           const uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
-          lb = v > lb ? v : lb;
+          if (v >= (uint64_t)S && xf == P) xf = x;
           fill += (uint64_t)divk(Fx, Kh, MK) + (uint64_t)divk(Cin, Kh, MK);
           tail += (uint64_t)wB[x];
         }
-        live = lb < (uint64_t)S;
+        live = xf == P;
+        if (!live && xf < P - 1) {
+          // LB_xf depends only on the prefix c_1..c_{xf+1}, so every partition with
+          // that prefix is pruned too: jump to the first lex partition after them (the
+          // lex successor restricted to positions <= xf+1) and re-rank it,
+          // rank = sum_x C(n-1-c_{x-1}, P-x) - C(n-c_x, P-x) (hockey-stick form of O7)
+          const int j = xf + 1;
+          int pos = 0;
+#pragma unroll
+          for (int x = P - 1; x >= 1; --x)
+            if (x <= j && pos == 0 && c[x] < n - (P - x)) pos = x;
+          if (pos == 0) break;  // no partition left in the whole space
+#pragma unroll
+          for (int x = 1; x <= P - 1; ++x) {
+            if (x == pos) c[x] = c[x] + 1;
+            else if (x > pos) c[x] = c[x - 1] + 1;
+          }
+          uint64_t nr = 0;
+#pragma unroll
+          for (int x = 1; x <= P - 1; ++x)
+            nr += binom_at(A.t.binom, n - 1 - c[x - 1], P - x) - binom_at(A.t.binom, n - c[x], P - x);
+          r = nr - 1;  // the loop's ++r lands on it
+          continue;
+        }
       }
       if (live && A.mode == 0) {
         for (int k = k_lo; k <= k_hi; ++k) {
@@ -2650,6 +2674,8 @@ static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int
     // kUnitsPerWarp units per warp so the end-of-kernel imbalance is ~1/kUnitsPerWarp
     // of a warp's work, while the per-unit unrank stays negligible
     uint64_t kUnitsPerWarp = 128, kMinSims = 128;
+    // pruned mode skips whole prefix blocks inside a lane's range: longer ranges
+    if (A.mode == 2) kUnitsPerWarp = 8;
     if (const char* e = getenv("AP_SWEEP_UPW")) kUnitsPerWarp = strtoull(e, nullptr, 10);
     if (const char* e = getenv("AP_SWEEP_MINSIMS")) kMinSims = strtoull(e, nullptr, 10);
     const uint64_t K = (uint64_t)(A.k_hi - A.k_lo + 1);

@@ -590,23 +590,32 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
         // (64-bit: m * load can exceed 2^32 for the heavy partitions it prunes)
         const uint32_t Kh = (uint32_t)k_hi, MK = s_mk[k_hi];
         uint64_t fill = 0, tail = 0;
-        int xf = P;  // first stage whose bound reaches S
+        int xf = P;        // first stage whose bound reaches S
+        bool mono = false;  // ... and does so without its comm terms
 #pragma unroll
         for (int x = 0; x < P; ++x) {
           const V Fx = sPf[c[x + 1]] - sPf[c[x]];
           const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
           const uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
-          if (v >= (uint64_t)S && xf == P) xf = x;
+          if (v >= (uint64_t)S && xf == P) {
+            xf = x;
+            const V Bx = sPb[c[x + 1]] - sPb[c[x]];
+            mono = fill + (uint64_t)m * ((uint64_t)Fx + (uint64_t)Bx) + tail >= (uint64_t)S;
+          }
           fill += (uint64_t)divk(Fx, Kh, MK) + (uint64_t)divk(Cin, Kh, MK);
           tail += (uint64_t)wB[x];
         }
         live = xf == P;
-        if (!live && xf < P - 1) {
+        if (!live && (xf < P - 1 || mono)) {
           // LB_xf depends only on the prefix c_1..c_{xf+1}, so every partition with
-          // that prefix is pruned too: jump to the first lex partition after them (the
-          // lex successor restricted to positions <= xf+1) and re-rank it,
+          // that prefix is pruned too.  If the bound holds on the stage's compute alone
+          // (fill and tail depend on c_1..c_xf; F_xf + B_xf grows with c_{xf+1}), every
+          // larger c_{xf+1} fails as well, and the prefix c_1..c_xf is done.  Jump to
+          // the first lex partition after the pruned block (the lex successor restricted
+          // to positions <= j) and re-rank it,
           // rank = sum_x C(n-1-c_{x-1}, P-x) - C(n-c_x, P-x) (hockey-stick form of O7)
-          const int j = xf + 1;
+          const int j = mono ? xf : xf + 1;
+          if (j == 0) break;  // stage 0 fails for this c_1 and every larger one
           int pos = 0;
 #pragma unroll
           for (int x = P - 1; x >= 1; --x)

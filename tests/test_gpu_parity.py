@@ -1031,3 +1031,30 @@ def test_eval_batch_fast_path(ap, oracle_mod, monkeypatch, mode):
         torch.cuda.synchronize()
         o = [M.simulate(p, m, list(c)) for c in cuts]
         assert T.tolist() == [x["T"] for x in o] and Mst.tolist() == [x["master"] for x in o], (mode, p, kind)
+
+
+def test_pruned_prefix_skips_random_windows(ap, oracle_mod):
+    """The pruned mode's prefix jumps (first failing stage bound, and its compute-only
+    monotone form) never skip a winner: on random problems and random rank windows the
+    key equals the full sweep's and the oracle's argmin over the same window."""
+    import torch
+    rng = np.random.default_rng(97)
+    for trial in range(40):
+        n = int(rng.integers(6, 22))
+        p = int(rng.integers(2, min(n, 8) + 1))
+        m = int(rng.integers(p, p + 10))
+        kind = ["b3f", "uniform", "huge", "small"][trial % 4]
+        f, b, a = synth.random_tables(1500 + trial, n, kind)
+        bw = synth.link_for(kind)
+        plan = _plan(ap, f, b, a, bw)
+        N = ap.ap_count(n, p)
+        lo = int(rng.integers(0, N))
+        hi = int(rng.integers(lo + 1, N + 1))
+        k_lo = int(rng.integers(1, 3)); k_hi = k_lo + int(rng.integers(0, 4))
+        k0 = _search_mode(ap, plan, p, m, k_lo, k_hi, 0, lo, hi)
+        k2 = _search_mode(ap, plan, p, m, k_lo, k_hi, 2, lo, hi)
+        assert k0 == k2, (trial, n, p, m, lo, hi)
+        if k0 != 0x7fffffffffffffff:
+            o = oracle_mod.Model(f, b, a, bw).exhaustive(p, m, k_lo, k_hi, lo, hi)
+            res = ap.ap_decode(plan, 0, p, m, k_lo, k_hi, key=k0)
+            assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])

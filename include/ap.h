@@ -203,6 +203,24 @@ ap_status ap_search_exhaustive2(const ap_plan* plan, int32_t p, int32_t m, int32
                                 int64_t* out, ap_stream_t stream);
 
 /*
+ * ap_search_exhaustive_bounded -- ap_search_exhaustive2 with a caller-supplied bound:
+ * only candidates with T <= min(T_ref, t_bound) are kept (the same u32 saturation and,
+ * in AP_SEARCH_PRUNED, the same lower-bound pruning, now at min(T_ref, t_bound) + 1).
+ * With t_bound an ATTAINED iteration time -- e.g. the heuristic's result
+ * (ap_search_heuristic) -- the global optimum T* <= t_bound is kept,
+ * so the reduced out over all shards is exactly the exhaustive argmin (SURVEY §8c O7,
+ * O11) while the pruning is as tight as the best plan already known.  With t_bound < T*
+ * every shard returns INT64_MAX.
+ *   t_bound  >= 0 (INVALID otherwise); INT64_MAX = ap_search_exhaustive2.
+ *   out      device int64[2], as ap_search_exhaustive2 (decode with ap_decode mode 2).
+ * Errors as ap_search_exhaustive2.
+ */
+ap_status ap_search_exhaustive_bounded(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                       int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
+                                       int32_t mode, int64_t t_bound, int64_t* out,
+                                       ap_stream_t stream);
+
+/*
  * ap_key2_select -- phase 2 of the two-phase reduction, stream-ordered on `stream`:
  * *idx = local[1] if local[0] == *t_star (and is not INT64_MAX), else INT64_MAX.
  *   local  device int64[2] from ap_search_exhaustive2; t_star, idx device int64[1].

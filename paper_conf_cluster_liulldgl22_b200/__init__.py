@@ -93,6 +93,8 @@ def _load_lib():
     lib.ap_alg1.argtypes = [vp, i32, P(i32), P(i64)]
     lib.ap_search_exhaustive2.restype = i32
     lib.ap_search_exhaustive2.argtypes = [vp, i32, i32, i32, i32, u64, u64, i32, vp, vp]
+    lib.ap_search_exhaustive_bounded.restype = i32
+    lib.ap_search_exhaustive_bounded.argtypes = [vp, i32, i32, i32, i32, u64, u64, i32, i64, vp, vp]
     lib.ap_key2_select.restype = i32
     lib.ap_key2_select.argtypes = [vp, vp, vp, vp]
     lib.ap_search_reachable.restype = i32
@@ -120,7 +122,7 @@ lib = _load_lib()
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
            "ap_plan_set_memory",
            "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_exhaustive_mode",
-           "ap_search_exhaustive2", "ap_key2_select",
+           "ap_search_exhaustive2", "ap_search_exhaustive_bounded", "ap_key2_select",
            "ap_search_heuristic", "ap_search_reachable", "ap_decode_reachable",
            "ap_last_truncated",
            "ap_decode", "ap_slice_sweep", "ap_slice_sweep_paper", "ap_slicer_alg2",
@@ -260,6 +262,14 @@ def ap_search_exhaustive2(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank
     _check(lib.ap_search_exhaustive2(plan.handle, int(p), int(m), int(k_lo), int(k_hi),
                                      int(rank_lo), int(rank_hi), int(mode),
                                      _ptr(out, "int64", plan.device, 2), _stream(stream)))
+
+
+def ap_search_exhaustive_bounded(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank_lo: int,
+                                 rank_hi: int, mode: int, t_bound: int, out, stream=None):
+    """ap_search_exhaustive2 keeping only T <= min(T_ref, t_bound) (t_bound attained)."""
+    _check(lib.ap_search_exhaustive_bounded(plan.handle, int(p), int(m), int(k_lo), int(k_hi),
+                                            int(rank_lo), int(rank_hi), int(mode), int(t_bound),
+                                            _ptr(out, "int64", plan.device, 2), _stream(stream)))
 
 
 def ap_key2_select(local, t_star, idx, stream=None):

@@ -596,7 +596,8 @@ namespace {
 // Shared by the packed-key and the two-phase entry points: exactly one of key / out2.
 ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
                                  int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int32_t mode,
-                                 int64_t* key, int64_t* out2, ap_stream_t stream) {
+                                 int64_t* key, int64_t* out2, ap_stream_t stream,
+                                 int64_t t_bound = INT64_MAX) {
   g_err.clear();
   const bool mem = (mode == AP_SEARCH_MEMORY);
   if (!mem && (mode < AP_SEARCH_FULL || mode > AP_SEARCH_PRUNED))
@@ -642,6 +643,7 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
                                   (unsigned __int128)2 * m * (p - 1) * (uint64_t)plan->max_comm;
     tref = (int64_t)tot;
   }
+  if (t_bound < tref) tref = t_bound;  // caller's attained bound (ap_search_exhaustive_bounded)
   if (key && (rb >= 63 || (uint64_t)tref >= ((1ull << (63 - rb)) - 1)))
     return fail(AP_ERR_RANGE, "key packing: T_ref=%lld needs %d bits + %d rank bits > 63",
                 (long long)tref, bitlen((unsigned __int128)tref), rb);
@@ -771,6 +773,17 @@ ap_status ap_search_exhaustive2(const ap_plan* plan, int32_t p, int32_t m, int32
   }
   return search_exhaustive_impl(plan, p, m, k_lo, k_hi, rank_lo, rank_hi, mode, nullptr, out,
                                 stream);
+}
+
+ap_status ap_search_exhaustive_bounded(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
+                                       int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
+                                       int32_t mode, int64_t t_bound, int64_t* out,
+                                       ap_stream_t stream) {
+  g_err.clear();
+  if (!out) return fail(AP_ERR_INVALID, "out is NULL");
+  if (t_bound < 0) return fail(AP_ERR_INVALID, "t_bound %lld < 0", (long long)t_bound);
+  return search_exhaustive_impl(plan, p, m, k_lo, k_hi, rank_lo, rank_hi, mode, nullptr, out,
+                                stream, t_bound);
 }
 
 ap_status ap_key2_select(const int64_t* local, const int64_t* t_star, int64_t* idx,

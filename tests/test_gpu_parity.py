@@ -1058,3 +1058,38 @@ def test_pruned_prefix_skips_random_windows(ap, oracle_mod):
             o = oracle_mod.Model(f, b, a, bw).exhaustive(p, m, k_lo, k_hi, lo, hi)
             res = ap.ap_decode(plan, 0, p, m, k_lo, k_hi, key=k0)
             assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"])
+
+
+def test_exhaustive_bounded(ap, oracle_mod):
+    """ap_search_exhaustive_bounded: with t_bound = an attained T >= the optimum (the
+    heuristic's, or the optimum itself) every mode returns the oracle's argmin; with
+    t_bound = optimum - 1 every shard is empty."""
+    import torch
+    rng = np.random.default_rng(41)
+    out = torch.empty(2, dtype=torch.int64, device="cuda")
+    hk = torch.empty(1, dtype=torch.int64, device="cuda")
+    for trial in range(12):
+        n = int(rng.integers(6, 20))
+        p = int(rng.integers(2, min(n, 8) + 1))
+        m = int(rng.integers(p, p + 8))
+        kind = ["b3f", "uniform", "equal"][trial % 3]
+        f, b, a = synth.random_tables(1700 + trial, n, kind)
+        bw = synth.link_for(kind)
+        plan = _plan(ap, f, b, a, bw)
+        N = ap.ap_count(n, p)
+        o = oracle_mod.Model(f, b, a, bw).exhaustive(p, m, 1, 2)
+        ap.ap_search_heuristic(plan, p, m, 0x5EED, 2, 0, 64, 0, hk)
+        torch.cuda.synchronize()
+        th = int(hk.item()) >> 20
+        for bound in (th, o["T"]):
+            for mode in (0, 1, 2):
+                ap.ap_search_exhaustive_bounded(plan, p, m, 1, 2, 0, N, mode, bound, out)
+                torch.cuda.synchronize()
+                res = ap.ap_decode(plan, 2, p, m, 1, 2, key=int(out[1].item()))
+                assert int(out[0].item()) == o["T"]
+                assert (res["time_ns"], res["rank"], res["k"]) == (o["T"], o["rank"], o["k"]), (trial, mode)
+        ap.ap_search_exhaustive_bounded(plan, p, m, 1, 2, 0, N, 2, o["T"] - 1, out)
+        torch.cuda.synchronize()
+        assert out.tolist() == [2**63 - 1, 2**63 - 1]
+    with pytest.raises(ap.APError):
+        ap.ap_search_exhaustive_bounded(plan, p, m, 1, 2, 0, N, 2, -1, out)

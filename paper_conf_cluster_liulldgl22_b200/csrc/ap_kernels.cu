@@ -596,7 +596,19 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
         for (int x = 0; x < P; ++x) {
           const V Fx = sPf[c[x + 1]] - sPf[c[x]];
           const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
-          const uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
+          uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
+          if (x < P - 1) {
+            // 1F1B bubble: B(x, 0) waits for micro-batch 0's round trip
+            // through the later stages, R = sum_{i>x} (split(F_i,k,k-1) + B_i) >=
+            // floor(sum_{i>x} F_i / K) - (P-1-x) + sum_{i>x} B_i (comms dropped, so R
+            // depends on c_{x+1} only), while the stage itself has only w_x = P-1-x
+            // forwards to run before it: T >= LB_x + max(0, R - w_x * wF_x).
+            const V Rf = sPf[n] - sPf[c[x + 1]], Rb = sPb[n] - sPb[c[x + 1]];
+            const uint64_t q = (uint64_t)divk(Rf, Kh, MK), w = (uint64_t)(P - 1 - x);
+            const uint64_t R = (Kh == 1 ? q : (q > w ? q - w : 0)) + (uint64_t)Rb;
+            const uint64_t own = w * (uint64_t)wF[x];
+            if (R > own) v += R - own;
+          }
           if (v >= (uint64_t)S && xf == P) {
             xf = x;
             const V Bx = sPb[c[x + 1]] - sPb[c[x]];

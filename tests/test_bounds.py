@@ -1,0 +1,54 @@
+"""CPU pin of the bound the GPU pruned search uses: SURVEY O11's chain
+bound plus the 1F1B bubble term, written out here from the DAG argument and checked to
+never exceed the oracle's exact T (like P6 for O11), for every k <= K.  It is a
+lower-bound formula only, so if it overshot, the pruned search could drop the optimum;
+this test (and the GPU key-equality tests) would catch that."""
+import numpy as np
+import pytest
+
+import synth
+
+
+def _bubble_bound(f, b, comm, n, p, m, K, cuts):
+    """max over stages x of: fill_x + m*(wF_x + wB_x) + tail_x
+    + max(0, R_x - (p-1-x)*wF_x), R_x = floor(sum_{i>x} F_i / K) - (p-1-x) [K > 1]
+    + sum_{i>x} B_i; wF_x = F_x + C_{x-1}, wB_x = B_x + C_x (receiver-side comm)."""
+    e = [0] + list(cuts) + [n]
+    F = [int(f[e[x]:e[x + 1]].sum()) for x in range(p)]
+    B = [int(b[e[x]:e[x + 1]].sum()) for x in range(p)]
+    C = [int(comm[e[x + 1] - 1]) if x < p - 1 else 0 for x in range(p)]
+    wF = [F[x] + (C[x - 1] if x > 0 else 0) for x in range(p)]
+    wB = [B[x] + C[x] for x in range(p)]
+    best = 0
+    fill = tail = 0
+    for x in range(p):
+        v = fill + m * (wF[x] + wB[x]) + tail
+        if x < p - 1:
+            w = p - 1 - x
+            q = sum(F[x + 1:]) // K
+            R = (q if K == 1 else max(q - w, 0)) + sum(B[x + 1:])
+            v += max(0, R - w * wF[x])
+        best = max(best, v)
+        fill += F[x] // K + (C[x - 1] // K if x > 0 else 0)
+        tail += wB[x]
+    return best
+
+
+def test_bubble_bound_never_exceeds_T(oracle_mod):
+    tight = stronger = 0
+    for seed in range(400):
+        kind = ["uniform", "b3f", "huge", "small", "equal"][seed % 5]
+        n = 5 + seed % 14
+        f, b, a = synth.random_tables(3000 + seed, n, kind)
+        bw = synth.link_for(kind)
+        M = oracle_mod.Model(f, b, a, bw)
+        p = 2 + seed % min(n - 1, 7)
+        m = p + seed % 6          # the pruned kernel runs with m >= p
+        K = 1 + seed % 4
+        cuts = synth.random_cuts(seed + 7, n, p, 1)[0]
+        lb = _bubble_bound(f, b, M.comm, n, p, m, K, cuts)
+        for k in range(1, K + 1):
+            assert M.T(p, m, cuts, k=k) >= lb, (seed, n, p, m, K, k)
+        stronger += lb > M.lower_bound(p, m, K, cuts)
+        tight += M.T(p, m, cuts, k=1) == lb
+    assert stronger > 0 and tight > 0

@@ -52,3 +52,28 @@ def test_bubble_bound_never_exceeds_T(oracle_mod):
         stronger += lb > M.lower_bound(p, m, K, cuts)
         tight += M.T(p, m, cuts, k=1) == lb
     assert stronger > 0 and tight > 0
+
+
+def test_bubble_bound_balanced_and_configs(oracle_mod):
+    """Near-balanced partitions (restart starts around Algorithm 1, where the bubble term
+    matters most) on random tables and on the five configs' tables: never above T."""
+    cases = []
+    for seed in range(60):
+        kind = ["uniform", "b3f", "equal"][seed % 3]
+        n = 10 + seed % 20
+        f, b, a = synth.random_tables(3500 + seed, n, kind)
+        cases.append((f, b, a, synth.link_for(kind), 2 + seed % 7, None, 1 + seed % 4))
+    for cfg in (1, 2, 3, 4, 5):
+        wl = synth.config(cfg)
+        f, b, a = wl.arrays()
+        cases.append((f, b, a, wl.link_bytes_per_s, wl.p, wl.m, max(wl.k_hi, 1)))
+    for f, b, a, bw, p, m, K in cases:
+        n = len(f)
+        p = min(p, n)
+        m = m or p + 3
+        M = oracle_mod.Model(f, b, a, bw)
+        for r in range(6):
+            cuts = [int(x) for x in M.restart_start(p, 0x5EED, 2, r)]
+            lb = _bubble_bound(f, b, M.comm, n, p, m, K, cuts)
+            for k in sorted({1, K}):
+                assert M.T(p, m, cuts, k=k) >= lb, (n, p, m, K, k, cuts)

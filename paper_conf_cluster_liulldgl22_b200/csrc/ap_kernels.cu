@@ -2696,7 +2696,7 @@ static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int
     // of a warp's work, while the per-unit unrank stays negligible
     uint64_t kUnitsPerWarp = 128, kMinSims = 128;
     // pruned mode skips whole prefix blocks inside a lane's range: longer ranges
-    if (A.mode == 2) kUnitsPerWarp = 8;
+    if (A.mode == 2) kUnitsPerWarp = 16;  // A/B: profiles/r01_pruned_upw.txt
     if (const char* e = getenv("AP_SWEEP_UPW")) kUnitsPerWarp = strtoull(e, nullptr, 10);
     if (const char* e = getenv("AP_SWEEP_MINSIMS")) kMinSims = strtoull(e, nullptr, 10);
     const uint64_t K = (uint64_t)(A.k_hi - A.k_lo + 1);

@@ -139,8 +139,8 @@ ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t
  * writes ONE packed int64 key to device memory:
  *     key = T << rb | (rank*(k_hi-k_lo+1) + k - k_lo),  rb = bitlen(N*K - 1),
  * N = C(n-1,p-1), K = k_hi-k_lo+1, or INT64_MAX if the slice holds no candidate
- * with T < T_ref+1, where T_ref = T(Algorithm 1 partition, k_lo)
- * is an attained upper bound on the optimum.  The minimum key over all slices is
+ * with T < T_ref+1, where T_ref = min over k in [k_lo, k_hi] of T(Algorithm 1
+ * partition, k) is an attained upper bound on the optimum.  The minimum key over all slices is
  * the lexicographic min of (T, rank, k) ("Return the partition scheme
  * with minimum iteration time"; reading Q15), so the keys of disjoint slices on
  * different GPUs combine with one all_reduce(MIN) (BASELINE north_star).
@@ -176,7 +176,7 @@ ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_
  * partitions that fit the plan's memory model (ap_plan_set_memory; INVALID without it):
  * every stage x must satisfy  sum(static) + min(p-x, m) * sum(stash) <= cap  over its
  * sub-layers (min(p-x, m) = the micro-batches 1F1B keeps in flight on stage x).  Runs
- * on the generic exact kernel.  T_ref is the Alg.-1 partition's T when that partition
+ * on the generic exact kernel.  T_ref is the Alg.-1 partition's T at k_lo when it
  * fits, else the overflow guard's bound on any T (then the packed key usually does not
  * fit and ap_search_exhaustive2 applies).  INT64_MAX when nothing fits. */
 #define AP_SEARCH_MEMORY 4
@@ -391,7 +391,7 @@ typedef struct {
   int32_t exact_p;         /* 1: kernel specialised for this p, 0: generic        */
   int32_t blocks, threads; /* grid                                                */
   uint64_t chunk;          /* ranks per thread                                    */
-  int64_t t_ref;           /* T(Algorithm 1 partition, k_lo)                      */
+  int64_t t_ref;           /* min_k T(Algorithm 1 partition, k), k in [k_lo,k_hi] */
   int32_t rank_bits;       /* rb                                                  */
   int32_t launches;        /* kernels launched by the call                        */
   int32_t clamp_rows;      /* u32 path: steady rows between saturating clamps      */

@@ -625,17 +625,24 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   int64_t* d_val;
   st = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
   if (st != AP_OK) return st;
+  // T_ref = min over k in [k_lo, k_hi] of T(Alg.-1 partition, k): an attained T, so the
+  // argmin has T <= T_ref (the memory mode keeps k_lo: its feasibility test is per plan)
+  const int nk = mem ? 1 : k_hi - k_lo + 1;
   int64_t* d_tref;
-  AP_CUDA(sc.get((void**)&d_tref, 8));
+  AP_CUDA(sc.get((void**)&d_tref, 8 * (size_t)nk));
   int launches = 1;
-  AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 0, 1,
+  AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 1, nk,
                            d_tref, nullptr, s, &launches));
-  int64_t tref = 0;
+  int64_t trefs[AP_MAX_K];
   int32_t a1h[32] = {0};
-  AP_CUDA(cudaMemcpyAsync(&tref, d_tref, 8, cudaMemcpyDeviceToHost, s));
+  AP_CUDA(cudaMemcpyAsync(trefs, d_tref, 8 * (size_t)nk, cudaMemcpyDeviceToHost, s));
   if (mem && p > 1) AP_CUDA(cudaMemcpyAsync(a1h, d_a1, 4 * (size_t)(p - 1), cudaMemcpyDeviceToHost, s));
   AP_CUDA(cudaStreamSynchronize(s));
-  if (tref < 0) return fail(AP_ERR_CUDA, "T_ref evaluation failed");
+  int64_t tref = trefs[0];
+  for (int i = 0; i < nk; ++i) {
+    if (trefs[i] < 0) return fail(AP_ERR_CUDA, "T_ref evaluation failed");
+    if (trefs[i] < tref) tref = trefs[i];
+  }
   if (mem && !plan->feasible(p, m, a1h)) {
     // the Alg.-1 partition does not fit: no attained feasible T to bound the search
     // with, so every candidate stays (S = the overflow guard's bound on any T)

@@ -592,10 +592,12 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
         uint64_t fill = 0, tail = 0;
         int xf = P;        // first stage whose bound reaches S
         bool mono = false;  // ... and does so without its comm terms
+        uint64_t alast = 0;  // the last stage's bound terms that do not depend on c_{P-1}
 #pragma unroll
         for (int x = 0; x < P; ++x) {
           const V Fx = sPf[c[x + 1]] - sPf[c[x]];
           const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
+          if (x == P - 2) alast = fill + (uint64_t)divk(Cin, Kh, MK) + tail;
           uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
           if (x < P - 1) {
             // 1F1B bubble: B(x, 0) waits for micro-batch 0's round trip
@@ -618,6 +620,35 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
           tail += (uint64_t)wB[x];
         }
         live = xf == P;
+        if (P >= 2 && xf == P - 1) {
+          // Only the last stage fails.  Its bound without the comm terms C_{P-2},
+          // L(c) = alast + floor((Pf[c]-Pf[c_{P-2}])/K) + Pb[c]-Pb[c_{P-2}]
+          //        + m*(Pf[n]-Pf[c] + Pb[n]-Pb[c]),  c = c_{P-1},
+          // is <= LB_{P-1} and non-increasing in c (one more sub-layer (f,b) adds at most
+          // f + b and removes m*(f+b)), so the failing c form a prefix of [c_{P-2}+1, n-1]:
+          // step c_{P-1} past it in shared memory instead of one rank at a time.
+          const int cl = c[P - 2];
+          auto L = [&](int cc) -> uint64_t {
+            return alast + (uint64_t)divk(V(sPf[cc] - sPf[cl]), Kh, MK) + (uint64_t)(sPb[cc] - sPb[cl]) +
+                   (uint64_t)m * ((uint64_t)(sPf[n] - sPf[cc]) + (uint64_t)(sPb[n] - sPb[cc]));
+          };
+          int cc = c[P - 1];
+          if (L(cc) >= (uint64_t)S) {
+            do ++cc; while (cc <= n - 1 && L(cc) >= (uint64_t)S);
+            if (cc <= n - 1) {
+              c[P - 1] = cc;
+              uint64_t nr = 0;
+#pragma unroll
+              for (int x = 1; x <= P - 1; ++x)
+                nr += binom_at(A.t.binom, n - 1 - c[x - 1], P - x) - binom_at(A.t.binom, n - c[x], P - x);
+              r = nr - 1;
+              continue;
+            }
+            // every c_{P-1} left fails: the prefix c_1..c_{P-2} is done
+            xf = P - 2;
+            mono = true;
+          }
+        }
         if (!live && (xf < P - 1 || mono)) {
           // LB_xf depends only on the prefix c_1..c_{xf+1}, so every partition with
           // that prefix is pruned too.  If the bound holds on the stage's compute alone

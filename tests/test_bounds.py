@@ -77,3 +77,36 @@ def test_bubble_bound_balanced_and_configs(oracle_mod):
             lb = _bubble_bound(f, b, M.comm, n, p, m, K, cuts)
             for k in sorted({1, K}):
                 assert M.T(p, m, cuts, k=k) >= lb, (n, p, m, K, k, cuts)
+
+
+def _last_stage_bound(f, b, comm, n, p, m, K, cuts):
+    """The last-stage skip's bound: stage p-1's chain bound
+    fill + m*(wF + wB) + tail with every C_{p-2} term dropped (the comm into the last
+    stage, in wF_{p-1} and in tail); the other comms depend on c_1..c_{p-2} only."""
+    e = [0] + list(cuts) + [n]
+    F = [int(f[e[x]:e[x + 1]].sum()) for x in range(p)]
+    B = [int(b[e[x]:e[x + 1]].sum()) for x in range(p)]
+    C = [int(comm[e[x + 1] - 1]) for x in range(p - 1)]
+    fill = sum(F[x] // K for x in range(p - 1)) + sum(C[x - 1] // K for x in range(1, p - 1))
+    tail = sum(B[:p - 1]) + sum(C[:p - 2])
+    return fill + m * (F[p - 1] + B[p - 1]) + tail
+
+
+def test_last_stage_bound_below_T_and_monotone(oracle_mod):
+    """Never above the oracle's T for any k <= K (the skip drops only candidates with
+    L >= S > T_opt), and non-increasing in c_{p-1} with c_1..c_{p-2} fixed (so the failing
+    c_{p-1} form a prefix of their range, which the kernel steps past)."""
+    for seed in range(300):
+        kind = ["uniform", "b3f", "huge", "small", "equal"][seed % 5]
+        n = 5 + seed % 14
+        f, b, a = synth.random_tables(5000 + seed, n, kind)
+        M = oracle_mod.Model(f, b, a, synth.link_for(kind))
+        p = 2 + seed % min(n - 1, 7)
+        m = p + seed % 6
+        K = 1 + seed % 4
+        cuts = [int(x) for x in synth.random_cuts(seed + 11, n, p, 1)[0]]
+        for k in range(1, K + 1):
+            assert M.T(p, m, cuts, k=k) >= _last_stage_bound(f, b, M.comm, n, p, m, K, cuts), seed
+        lo = cuts[-2] + 1 if p > 2 else 1
+        seq = [_last_stage_bound(f, b, M.comm, n, p, m, K, cuts[:-1] + [c]) for c in range(lo, n)]
+        assert all(x >= y for x, y in zip(seq, seq[1:])), (seed, seq)

@@ -253,9 +253,15 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         if args.backend == "nccl":
+            # communicator-init logging stays on (stderr), so a scaling run shows every
+            # rank joining the NCCL communicator
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
             dist.init_process_group("nccl", device_id=dev)
         else:
             dist.init_process_group("gloo")
+        print(f"[bench] rank {rank}/{world} backend {args.backend} on cuda:{local}",
+              file=sys.stderr, flush=True)
     peaks, peak_src = _peaks()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
     sms = torch.cuda.get_device_properties(local).multi_processor_count

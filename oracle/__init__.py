@@ -111,6 +111,9 @@ def _load():
                                                  i32, i32, P(i64), P(i32)]
             lib.or_alg2.restype = i32
             lib.or_alg2.argtypes = [i32, P(i64), P(i64), P(i64), i32, P(i32), i32, P(i32)]
+            lib.or_alg2_trace.restype = i32
+            lib.or_alg2_trace.argtypes = [i32, P(i64), P(i64), P(i64), i32, P(i32), i32, P(i32),
+                                          P(i64), P(i64), P(i64)]
             lib.or_slice_sweep.restype = i32
             lib.or_slice_sweep.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, P(i32), i32,
                                            P(i64), P(i32)]
@@ -418,8 +421,27 @@ def _alg2(self, p, cuts, reading=0):
     return mb.value
 
 
+def _alg2_trace(self, p, cuts, reading=0):
+    """Algorithm 2 with its state recorded (see or_alg2_trace): returns
+    (mb, startt[p], [endt rows per pass], [tempt per pass])."""
+    lib = _load()
+    c = _i32(cuts) if p > 1 else np.zeros(1, np.int32)
+    mb = C.c_int32()
+    st = np.zeros(p, np.int64)
+    en = np.zeros(p * (p + 1) * 2, np.int64)
+    te = np.zeros(p, np.int64)
+    _chk(lib.or_alg2_trace(self.n, _p(self.f, C.c_int64), _p(self.b, C.c_int64),
+                           _p(self.comm, C.c_int64), p, _p(c, C.c_int32), reading, C.byref(mb),
+                           _p(st, C.c_int64), _p(en, C.c_int64), _p(te, C.c_int64)))
+    en = en.reshape(p, p + 1, 2)
+    return (mb.value, [int(x) for x in st],
+            [[[int(v) for v in row] for row in en[i]] for i in range(mb.value)],
+            [int(x) for x in te[: mb.value]])
+
+
 Model.slice_sweep_paper = _slice_paper
 Model.alg2 = _alg2
+Model.alg2_trace = _alg2_trace
 
 
 def count(n: int, p: int) -> int:

@@ -86,14 +86,20 @@ def search_exhaustive(plan: Plan, p: int, m: int, k_lo: int = 1, k_hi: int = 1,
                       two_phase: Optional[bool] = None, mode: int = 0) -> dict:
     """Exact argmin over all C(n-1,p-1) partitions x k in [k_lo,k_hi], sharded over
     the ranks of the default process group (if initialised).  two_phase None: the
-    packed key when it fits, else the two-phase reduction (every rank takes the same
-    branch: T_ref is the same global value on all of them)."""
+    packed key when it fits, else the two-phase reduction.  Every rank takes the same
+    branch: the packing test depends only on T_ref and N (global values), and when
+    N < world (an empty shard, which cannot run the test) the two-phase form is used
+    on every rank.""" 
     rank, world, dist = _world()
     N = ap_count(plan.n, p)
     lo, hi = shard(N, rank, world)
     dev = f"cuda:{plan.device}"
     out = {"sims": (hi - lo) * (k_hi - k_lo + 1), "total_sims": N * (k_hi - k_lo + 1),
            "shard": (lo, hi), "two_phase": False}
+    if two_phase is None and N < world:
+        # some rank has an empty shard and never learns whether the packed key fits;
+        # decide without it (the same on every rank): the two-phase form always fits
+        two_phase = True
     if not two_phase:
         key = torch.empty(1, dtype=torch.int64, device=dev)
         try:

@@ -9,11 +9,13 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libap.so")
 SOURCES = ["ap_kernels.cu", "ap_host.cu"]
-HEADERS = ["ap_device.cuh", "ap_launch.h", os.path.join("..", "..", "include", "ap.h")]
+HEADERS = ["ap_device.cuh", "ap_launch.h", "ap_master.cuh", os.path.join("..", "..", "include", "ap.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
-         "-cudart", "shared"]
+         "-cudart", "shared",
+         # the kernels' device code compiles in parallel, one kernel per job
+         "--split-compile", str(max(1, min(16, os.cpu_count() or 1)))]
 
 
 def _stale() -> bool:

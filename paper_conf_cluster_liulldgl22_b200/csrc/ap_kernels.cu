@@ -20,6 +20,7 @@
 
 #include "ap_device.cuh"
 #include "ap_launch.h"
+#include "ap_master.cuh"
 
 namespace apk {
 using namespace apdev;
@@ -1074,10 +1075,11 @@ struct EvalArgs {
   // redo pass (fastS = 0, redo_in set): evaluates exactly the listed candidates
   unsigned int* redo;
   const unsigned int* redo_in;
+  uint32_t one;     // = 1, opaque to the compiler (keeps the adds on IMAD)
 };
-// u32 copies of the prefix sums / comm and the floor(v/k) magics for the fast path
+// u32 copies of the prefix sums Pf, Pb, the comm and the floor(v/k) magics (fast path)
 __host__ __device__ inline size_t eval_fast_smem(int n) {
-  return ((size_t)(2 * n + 1 + kMaxK + 1) * 4 + 15) & ~size_t(15);
+  return ((size_t)(3 * n + 2 + kMaxK + 1) * 4 + 15) & ~size_t(15);
 }
 
 template <int P>
@@ -1101,26 +1103,12 @@ AP_DEV_INLINE bool load_cuts(const int32_t* row, int p, int n, int (&c)[P + 1]) 
 
 template <int P>
 __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
+  // the generic exact int64 evaluation (any p <= P, m, k, s); with A.redo_in set it
+  // evaluates exactly the candidates k_eval_fast listed
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
-  size_t off = (used + 15) & ~size_t(15);
-  uint32_t *s32Pf = nullptr, *s32C = nullptr, *s32mk = nullptr;
-  if (A.fastS) {  // block-uniform
-    s32Pf = reinterpret_cast<uint32_t*>(smem + off);
-    s32C = s32Pf + (A.t.n + 1);
-    s32mk = s32C + A.t.n;
-    for (int e = threadIdx.x; e <= A.t.n; e += blockDim.x) {
-      s32Pf[e] = (uint32_t)T.Pf[e];
-      if (e < A.t.n) s32C[e] = (uint32_t)T.comm[e];
-    }
-    if (threadIdx.x <= kMaxK)
-      s32mk[threadIdx.x] = (threadIdx.x <= 1) ? 0xffffffffu
-                           : A.div1 ? (uint32_t)(((1ull << 32) + threadIdx.x - 1) / threadIdx.x)
-                                    : (uint32_t)((1ull << 32) / threadIdx.x);
-    off += eval_fast_smem(A.t.n);
-    __syncthreads();
-  }
+  const size_t off = (used + 15) & ~size_t(15);
   const int p = A.p, m = A.m, n = A.t.n;
   // grid-stride (persistent) loop: the table prologue above runs once per CTA
   const int64_t cnt = A.redo_in ? (int64_t)A.redo_in[0] : A.count;
@@ -1146,57 +1134,90 @@ __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
     }
     uint32_t pb[P];
     TimesRef not_{nullptr, nullptr, nullptr};
-    BitsRef br{nullptr, 0};
-    if (A.master) {
-      if (A.gbits) {
-        br.base = A.gbits + i;
-        br.stride = (int)A.count;
-      } else {
-        uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + off);
-        br.base = sbits + threadIdx.x;
-        br.stride = blockDim.x;
-      }
-    }
-    if constexpr (P >= 2 && P <= 16) {
-      // u32 fast path: the N-form sweep (T only) or the M-form with decision bits and
-      // the branch-free backtrack (k = 1); exact below fastS
-      if (A.fastS && p == P && m >= P && m <= 32767) {
-        uint32_t wF[P], wB[P];
-  #pragma unroll
-        for (int x = 0; x < P; ++x) {
-          wF[x] = (uint32_t)(F[x] + ((x > 0) ? C[x - 1] : 0));
-          wB[x] = (uint32_t)(B[x] + C[x]);
-        }
-        if (A.master == nullptr) {
-          const ClampSched cs{0, A.CR, 1};
-          const uint32_t t32 = sim_fast<P, uint32_t>(m, k, wF, wB, c, s32Pf, s32C, s32mk[k],
-                                                     A.div1 != 0, A.fastS, cs, 1u);
-          if (t32 < A.fastS) {
-            A.time_ns[i] = (int64_t)t32;
-          } else {
-            A.redo[1 + atomicAdd(&A.redo[0], 1u)] = (unsigned int)i;
-          }
-          continue;
-        } else if (k == 1) {
-          const uint32_t t32 = sim_fast_bits<P>(m, wF, wB, A.fastS, A.CR, br);
-          if (t32 < A.fastS) {
-            A.time_ns[i] = (int64_t)t32;
-            A.master[i] = m <= 127 ? backtrack_master_bl<P, 8>(m, br) : backtrack_master_bl<P, 16>(m, br);
-          } else {
-            A.redo[1 + atomicAdd(&A.redo[0], 1u)] = (unsigned int)i;
-          }
-          continue;
-        }
-      }
-    }
     if (A.master == nullptr) {
       BitsRef nob{nullptr, 0};
       A.time_ns[i] = sim_exact<P, 0>(p, m, k, F, B, C, nob, pb, not_);
       continue;
     }
+    BitsRef br{nullptr, 0};
+    if (A.gbits) {
+      br.base = A.gbits + i;
+      br.stride = (int)A.count;
+    } else {
+      uint32_t* sbits = reinterpret_cast<uint32_t*>(smem + off);
+      br.base = sbits + threadIdx.x;
+      br.stride = blockDim.x;
+    }
     A.time_ns[i] = sim_exact<P, 1>(p, m, k, F, B, C, br, pb, not_);
     int len;
     A.master[i] = backtrack_master<P>(p, m, k, br, pb, &len, NoEmit{});
+  }
+}
+
+// K2 fast path (p == P <= 16, m >= P, micro-batch 0 sliced, u32 exact below fastS):
+// T for any k with the N-form sweep (sim_fast), T + master for k = 1, m <= 127 with
+// the recorded decision words and the run-length backtrack (ap_master.cuh).  Every
+// candidate it cannot finish exactly -- saturated at fastS, or T + master with k > 1
+// or m > 127 -- goes to A.redo for the generic k_eval.  A kernel of its own, so its
+// register allocation is not the generic path's.
+template <int P>
+__global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  size_t off = (used + 15) & ~size_t(15);
+  const int m = A.m, n = A.t.n;
+  uint32_t* s32Pf = reinterpret_cast<uint32_t*>(smem + off);
+  uint32_t* s32Pb = s32Pf + (n + 1);
+  uint32_t* s32C = s32Pb + (n + 1);
+  uint32_t* s32mk = s32C + n;
+  for (int e = threadIdx.x; e <= n; e += blockDim.x) {
+    s32Pf[e] = (uint32_t)T.Pf[e];
+    s32Pb[e] = (uint32_t)T.Pb[e];
+    if (e < n) s32C[e] = (uint32_t)T.comm[e];
+  }
+  if (threadIdx.x <= kMaxK)
+    s32mk[threadIdx.x] = (threadIdx.x <= 1) ? 0xffffffffu
+                         : A.div1 ? (uint32_t)(((1ull << 32) + threadIdx.x - 1) / threadIdx.x)
+                                  : (uint32_t)((1ull << 32) / threadIdx.x);
+  off += eval_fast_smem(n);
+  __syncthreads();
+  const Bits16 br{reinterpret_cast<uint16_t*>(smem + off) + threadIdx.x, (int)blockDim.x};
+  const uint32_t S = A.fastS, one = A.one;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < A.count;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    int c[P + 1];
+    const bool okc = load_cuts<P>(A.cuts + (size_t)i * A.cuts_stride, P, n, c);
+    const int k = A.kptr ? A.kptr[i] : (A.k_iota ? (int)(i + 1) : A.k_const);
+    if (!okc || k < 1 || k > kMaxK) {
+      A.time_ns[i] = -1;
+      if (A.master) A.master[i] = -1;
+      continue;
+    }
+    uint32_t wF[P], wB[P];
+#pragma unroll
+    for (int x = 0; x < P; ++x) {
+      wF[x] = (s32Pf[c[x + 1]] - s32Pf[c[x]]) + ((x > 0) ? s32C[c[x] - 1] : 0u);
+      wB[x] = (s32Pb[c[x + 1]] - s32Pb[c[x]]) + ((x < P - 1) ? s32C[c[x + 1] - 1] : 0u);
+    }
+    bool done = false;
+    if (A.master == nullptr) {
+      const ClampSched cs{0, A.CR, 1};
+      const uint32_t t32 = sim_fast<P, uint32_t>(m, k, wF, wB, c, s32Pf, s32C, s32mk[k],
+                                                 A.div1 != 0, S, cs, one);
+      if (t32 < S) {
+        A.time_ns[i] = (int64_t)t32;
+        done = true;
+      }
+    } else if (k == 1 && m <= 127) {
+      const uint32_t t32 = sim_bits16<P>(m, wF, wB, S, A.CR, br, one);
+      if (t32 < S) {
+        A.time_ns[i] = (int64_t)t32;
+        A.master[i] = backtrack_rows<P, 8>(m, br);
+        done = true;
+      }
+    }
+    if (!done) A.redo[1 + atomicAdd(&A.redo[0], 1u)] = (unsigned int)i;
   }
 }
 
@@ -1623,18 +1644,24 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
 }
 
 // ===========================================================================
-// K3p heuristic restarts as a per-CTA simulation pool (adjust_mode 0, u32 fast path,
-// p == P, m >= P).  In k_heur one lane owns one restart, so a warp
-// runs as long as its longest walk and its lanes simulate out of step.  Here a CTA
-// owns NS restart slots.  One thread per slot advances its walk (reading O9, in
-// exactly k_heur's order) and emits simulation jobs -- the start, or the up to four
-// children a, a', b, b' of a step -- into a shared-memory ring.  Every pass each of
-// the NT threads simulates one queued job, all in step.  A slot whose jobs are all
-// done advances at the next pass; free slots refill from the global restart cursor.
+// K3p heuristic restarts as WARP-OWNED simulation pools (adjust_mode 0, u32 fast path,
+// p == P <= 16, P <= m <= 127).  With one lane per restart (k_heur) a
+// warp runs as long as its longest walk and its lanes simulate out of step.  Here each
+// warp owns NSW restart slots: lane l < NSW advances slot l's walk (reading O9, in
+// exactly k_heur's order) and queues its simulation jobs -- the start, or the up to
+// four children a, a', b, b' of a step -- in the warp's ring; then each of the 32
+// lanes simulates one queued job (sim_bits16 + backtrack_rows, ap_master.cuh), all in
+// step.  A slot whose jobs are all done advances at the next pass; free slots refill
+// from the global restart cursor.  Only __syncwarp: the warps of a CTA never wait for
+// each other.
 namespace hpool {
-constexpr int NT = 256;   // threads per CTA = jobs simulated per pass
-constexpr int NS = 96;    // restart slots per CTA
-constexpr int RING = 512; // job ring, >= 4 * NS
+constexpr int NT = 128;   // threads per CTA (4 independent warp pools)
+constexpr int NW = NT / 32;
+#ifndef AP_HEUR_NSW
+#define AP_HEUR_NSW 24
+#endif
+constexpr int NSW = AP_HEUR_NSW;  // restart slots per warp (lanes 0..NSW-1 own them)
+constexpr int RING = 128;         // job ring per warp, >= 4 * NSW
 }  // namespace hpool
 
 // Child idx (0 a, 1 a', 2 b, 3 b') of `cur` with master i (
@@ -1668,7 +1695,7 @@ AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
 }
 
 template <int P>
-__global__ void __launch_bounds__(hpool::NT, 2) k_heur_pool(HeurArgs A) {
+__global__ void __launch_bounds__(hpool::NT, 4) k_heur_pool(HeurArgs A) {
   using namespace hpool;
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
@@ -1677,131 +1704,133 @@ __global__ void __launch_bounds__(hpool::NT, 2) k_heur_pool(HeurArgs A) {
   int16_t* s_arg = reinterpret_cast<int16_t*>(smem + ((used + 15) & ~size_t(15)));
   const int narg = (n + 1) * P1;
   int32_t* s_a1 = reinterpret_cast<int32_t*>(s_arg + ((narg + 7) & ~7));
-  uint32_t* s_bits = reinterpret_cast<uint32_t*>(s_a1 + 32);
-  // slot state: cut vectors [slot][0 cur | 1 best | 2+idx child idx][P+1]
-  __shared__ int16_t s_cuts[NS][6][P + 1];
-  __shared__ uint32_t s_chT[NS][4];
-  __shared__ int8_t s_chM[NS][4];
-  __shared__ uint32_t s_r[NS], s_bestT[NS];
-  __shared__ int s_pend[NS];
-  __shared__ int8_t s_state[NS], s_curM[NS], s_valid[NS], s_aband[NS];
-  __shared__ int s_steps[NS], s_nsims[NS];
-  __shared__ uint16_t s_ring[RING];
-  __shared__ int s_head, s_tail, s_stop;
-  const int tid = threadIdx.x;
+  uint32_t* s32Pf = reinterpret_cast<uint32_t*>(s_a1 + 32);
+  uint32_t* s32Pb = s32Pf + (n + 1);
+  uint32_t* s32C = s32Pb + (n + 1);
+  uint16_t* s_bits = reinterpret_cast<uint16_t*>(s32C + ((n + 3) & ~3));
+  // per-warp slot state: cut vectors [slot][0 cur | 1 best][P+1]; a job is a slot and a
+  // code (0-3: child a, a', b, b' of cur, 4: cur itself), and the lane that simulates it
+  // rebuilds the child in its own scratch vector (s_scr) from cur
+  __shared__ int16_t s_cuts[NW][NSW][2][P + 1];
+  static_assert(NSW <= 32 && 4 * NSW <= RING, "");
+  __shared__ int16_t s_scr[NW][32][P + 1];
+  __shared__ uint32_t s_chT[NW][NSW][4];
+  __shared__ int8_t s_chM[NW][NSW][4];
+  __shared__ int8_t s_curM[NW][NSW];
+  __shared__ int s_pend[NW][NSW];
+  __shared__ int8_t s_aband[NW][NSW];
+  __shared__ uint16_t s_ring[NW][2][RING];  // [0] walks past HOT steps, [1] the rest
+  const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   for (int e = tid; e < narg; e += NT) s_arg[e] = A.arg[e];
   for (int e = tid; e < p - 1; e += NT) s_a1[e] = A.alg1[e];
-  for (int s = tid; s < NS; s += NT) s_state[s] = 0;
-  if (tid == 0) {
-    s_head = 0;
-    s_tail = 0;
-    s_stop = 0;
+  for (int e = tid; e <= n; e += NT) {
+    s32Pf[e] = (uint32_t)T.Pf[e];
+    s32Pb[e] = (uint32_t)T.Pb[e];
+    if (e < n) s32C[e] = (uint32_t)T.comm[e];
   }
   __syncthreads();
-  const BitsRef br{s_bits + tid, NT};
+  const Bits16 br{s_bits + tid, NT};
+  int16_t* scr = s_scr[w][lane];
   const int smax = n * p;
+  const uint32_t one = A.CR > 0 ? 1u : 0u;  // = 1, not a compile-time constant
   unsigned long long my_key = 0x7fffffffffffffffull;
   unsigned int my_sims = 0;
+  // state of the slot owned by this lane (NSW = 32: one slot per lane), in registers
+  int st = 0, curM = 0, steps = 0, nsims = 0, valid = 0;
+  uint32_t r = 0, bestT = 0;
+  bool stop = false;
+  int head[2] = {0, 0}, tail[2] = {0, 0};  // warp-uniform ring cursors
+  // Walks are bimodal (C5: 80 % end within 8 steps, the rest take 21-29), and the last
+  // long walks set the kernel's length: the jobs of walks past HOT steps go first.
+  constexpr int HOT = 6;
+  const bool owner = lane < NSW;  // lanes 0..NSW-1 own one restart slot each
+  int16_t* cur = s_cuts[w][owner ? lane : 0][0];
+  int16_t* best = s_cuts[w][owner ? lane : 0][1];
 
   for (;;) {
-    // ---- phase A: advance the walks whose jobs are all done, refill free slots
-    if (tid < NS) {
-      const int s = tid;
-      int st = s_state[s];
-      if (st != 0 && s_pend[s] == 0) {
-        if (s_aband[s]) {
-          // a simulation saturated: the exact int64 pass redoes the whole restart
-          const unsigned int slot = atomicAdd(&A.redo[0], 1u);
-          A.redo[1 + slot] = s_r[s];
-          st = 0;
-        } else {
-          int16_t* cur = s_cuts[s][0];
-          int curM, steps, nsims;
-          uint32_t bestT;
-          bool walk = true;
-          if (st == 1) {  // the start was simulated
-            curM = s_chM[s][0];
-            bestT = s_chT[s][0];
-            for (int x = 0; x <= P; ++x) {
-              cur[x] = s_cuts[s][2][x];
-              s_cuts[s][1][x] = cur[x];
+    // ---- phase A: advance this lane's walk if its jobs are all done, refill if free
+    int nj = 0;
+    if (owner && st != 0 && s_pend[w][lane] == 0) {
+      if (s_aband[w][lane]) {
+        // a simulation saturated: the exact int64 pass redoes the whole restart
+        const unsigned int slot = atomicAdd(&A.redo[0], 1u);
+        A.redo[1 + slot] = r;
+        st = 0;
+      } else {
+        bool walk = true;
+        if (st == 1) {  // the start was simulated
+          curM = s_chM[w][lane][0];
+          bestT = s_chT[w][lane][0];
+          for (int x = 0; x <= P; ++x) best[x] = cur[x];
+          steps = 0;
+          nsims = 1;
+        } else {  // the children of a step were simulated: visit them in child order
+          uint32_t selT = 0xffffffffu;
+          int sel = -1, selM = 0;
+          for (int idx = 0; idx < 4; ++idx) {
+            if (!((valid >> idx) & 1)) continue;
+            ++nsims;
+            const uint32_t Tc = s_chT[w][lane][idx];
+            const int Mc = s_chM[w][lane][idx];
+            if (Tc < bestT) {
+              bestT = Tc;
+              pool_child(cur, idx, curM, p, P1, s_arg, scr);
+              for (int x = 0; x <= P; ++x) best[x] = scr[x];
             }
-            steps = 0;
-            nsims = 1;
-          } else {  // the children of a step were simulated: visit them in child order
-            curM = s_curM[s];
-            bestT = s_bestT[s];
-            steps = s_steps[s];
-            nsims = s_nsims[s];
-            const int valid = s_valid[s];
-            uint32_t selT = 0xffffffffu;
-            int sel = -1, selM = 0;
-            for (int idx = 0; idx < 4; ++idx) {
-              if (!((valid >> idx) & 1)) continue;
-              ++nsims;
-              const uint32_t Tc = s_chT[s][idx];
-              const int Mc = s_chM[s][idx];
-              if (Tc < bestT) {
-                bestT = Tc;
-                for (int x = 0; x <= P; ++x) s_cuts[s][1][x] = s_cuts[s][2 + idx][x];
-              }
-              if (Mc <= curM && Tc < selT) {
-                selT = Tc;
-                selM = Mc;
-                sel = idx;
-              }
-            }
-            if (sel < 0) {
-              walk = false;  // no child qualifies
-            } else {
-              for (int x = 0; x <= P; ++x) cur[x] = s_cuts[s][2 + sel][x];
-              curM = selM;
+            if (Mc <= curM && Tc < selT) {
+              selT = Tc;
+              selM = Mc;
+              sel = idx;
             }
           }
-          // next step (k_heur's begin_step with adjust_mode 0): the step cap, stop at
-          // master 0, else the children of step 3
-          int valid = 0, nj = 0;
-          if (walk && steps < smax && curM != 0) {
-            ++steps;
-            for (int idx = 0; idx < 4; ++idx)
-              if (pool_child(cur, idx, curM, p, P1, s_arg, s_cuts[s][2 + idx])) {
-                valid |= 1 << idx;
-                ++nj;
-              }
-          }
-          if (nj > 0) {
-            const int at = atomicAdd(&s_tail, nj);
-            int q = 0;
-            for (int idx = 0; idx < 4; ++idx)
-              if ((valid >> idx) & 1) s_ring[(at + q++) & (RING - 1)] = (uint16_t)(s * 4 + idx);
-            s_pend[s] = nj;
-            s_valid[s] = (int8_t)valid;
-            s_curM[s] = (int8_t)curM;
-            s_bestT[s] = bestT;
-            s_steps[s] = steps;
-            s_nsims[s] = nsims;
-            st = 2;
-          } else {  // the restart is finished
-            const uint32_t r = s_r[s];
-            my_sims += (unsigned int)nsims;
-            my_key = min(my_key, ((unsigned long long)bestT << 20) | r);
-            if (A.best_out)
-              for (int x = 1; x <= p - 1; ++x)
-                A.best_out[(size_t)(r - A.r_lo) * (p - 1) + (x - 1)] = s_cuts[s][1][x];
-            st = 0;
+          if (sel < 0) {
+            walk = false;  // no child qualifies
+          } else {
+            pool_child(cur, sel, curM, p, P1, s_arg, scr);
+            for (int x = 0; x <= P; ++x) cur[x] = scr[x];
+            curM = selM;
           }
         }
+        // next step (k_heur's begin_step with adjust_mode 0): the step cap, stop at
+        // master 0, else the children of step 3
+        valid = 0;
+        if (walk && steps < smax && curM != 0) {
+          ++steps;
+          for (int idx = 0; idx < 4; ++idx)
+            if (pool_child(cur, idx, curM, p, P1, s_arg, scr)) {
+              valid |= 1 << idx;
+              ++nj;
+            }
+        }
+        if (nj > 0) {
+          s_curM[w][lane] = (int8_t)curM;
+          st = 2;
+        } else {  // the restart is finished
+          my_sims += (unsigned int)nsims;
+          my_key = min(my_key, ((unsigned long long)bestT << 20) | r);
+          if (A.best_out)
+            for (int x = 1; x <= p - 1; ++x)
+              A.best_out[(size_t)(r - A.r_lo) * (p - 1) + (x - 1)] = best[x];
+          st = 0;
+        }
       }
-      // s_stop is written and read by several slot threads in the same phase: atomics
-      if (st == 0 && atomicAdd(&s_stop, 0) == 0) {
-        const uint32_t r = atomicAdd(A.counter, 1u) + A.r_lo;
+    }
+    // refill: one global atomic per warp for all its free slots
+    const bool want = owner && st == 0 && !stop;
+    const unsigned int wmask = __ballot_sync(0xffffffffu, want);
+    if (wmask) {
+      unsigned int base = 0;
+      if (lane == __ffs(wmask) - 1) base = atomicAdd(A.counter, (unsigned int)__popc(wmask));
+      base = __shfl_sync(0xffffffffu, base, __ffs(wmask) - 1);
+      if (want) {
+        r = base + (unsigned int)__popc(wmask & ((1u << lane) - 1u)) + A.r_lo;
         if (r >= A.r_hi) {
-          atomicOr(&s_stop, 1);
+          stop = true;
         } else {
           // restart start: Alg. 1 (r = 0) or the seeded perturbation (reading Q21)
           int prev = 0;
-          s_cuts[s][2][0] = 0;
-          s_cuts[s][2][P] = (int16_t)n;
+          cur[0] = 0;
+          cur[P] = (int16_t)n;
           for (int x = 1; x <= p - 1; ++x) {
             int64_t v = s_a1[x - 1];
             if (r != 0) {
@@ -1810,55 +1839,82 @@ __global__ void __launch_bounds__(hpool::NT, 2) k_heur_pool(HeurArgs A) {
               v = v < prev + 1 ? prev + 1 : v;
               v = v > n - (p - x) ? n - (p - x) : v;
             }
-            s_cuts[s][2][x] = (int16_t)v;
+            cur[x] = (int16_t)v;
             prev = (int)v;
           }
-          s_r[s] = r;
-          s_aband[s] = 0;
-          s_pend[s] = 1;
-          const int at = atomicAdd(&s_tail, 1);
-          s_ring[at & (RING - 1)] = (uint16_t)(s * 4);
+          s_aband[w][lane] = 0;
+          valid = 16;  // job code 4: cur itself
+          nj = 1;
           st = 1;
         }
       }
-      s_state[s] = (int8_t)st;
     }
-    if (!__syncthreads_or(tid < NS && s_state[tid] != 0)) break;
-    // ---- phase B: one queued job per thread, all simulated in step
-    const int head = s_head;
-    const int nj = min(s_tail - head, NT);
-    if (tid < nj) {
-      const int job = s_ring[(head + tid) & (RING - 1)];
-      const int s = job >> 2, idx = job & 3;
-      int cc[P + 1];
+    // stop: the cursor ran out for one lane, so it has for every later refill too
+    stop = __any_sync(0xffffffffu, stop);
+    // queue the jobs: warp prefix sums of nj per ring (no atomics)
+    const int hot = (st == 2 && steps >= HOT) ? 0 : 1;
+    int off0 = hot == 0 ? nj : 0, off1 = hot == 1 ? nj : 0;
 #pragma unroll
-      for (int x = 0; x <= P; ++x) cc[x] = s_cuts[s][2 + idx][x];
-      int64_t F[P], B[P], C[P];
-      stage_costs<P>(T, p, cc, F, B, C);
+    for (int o = 1; o < 32; o <<= 1) {
+      const int v0 = __shfl_up_sync(0xffffffffu, off0, o);
+      const int v1 = __shfl_up_sync(0xffffffffu, off1, o);
+      if (lane >= o) {
+        off0 += v0;
+        off1 += v1;
+      }
+    }
+    const int tot0 = __shfl_sync(0xffffffffu, off0, 31);
+    const int tot1 = __shfl_sync(0xffffffffu, off1, 31);
+    if (nj > 0) {
+      int q = tail[hot] + (hot == 0 ? off0 : off1) - nj;
+      for (int code = 0; code < 5; ++code)
+        if ((valid >> code) & 1) s_ring[w][hot][(q++) & (RING - 1)] = (uint16_t)(lane * 8 + code);
+      s_pend[w][lane] = nj;
+    }
+    tail[0] += tot0;
+    tail[1] += tot1;
+    if (!__any_sync(0xffffffffu, owner && st != 0)) break;
+    __syncwarp();
+    // ---- phase B: one queued job per lane, all simulated in step
+    const int nj0 = min(tail[0] - head[0], 32);
+    const int nj1 = min(tail[1] - head[1], 32 - nj0);
+    if (lane < nj0 + nj1) {
+      const int job = lane < nj0 ? s_ring[w][0][(head[0] + lane) & (RING - 1)]
+                                 : s_ring[w][1][(head[1] + lane - nj0) & (RING - 1)];
+      const int sl = job >> 3, code = job & 7;
+      const int16_t* src = s_cuts[w][sl][0];
+      if (code < 4) {
+        pool_child(src, code, s_curM[w][sl], p, P1, s_arg, scr);
+        src = scr;
+      }
+      int c[P + 1];
+#pragma unroll
+      for (int x = 0; x <= P; ++x) c[x] = src[x];
       uint32_t wF[P], wB[P];
 #pragma unroll
       for (int x = 0; x < P; ++x) {
-        wF[x] = (uint32_t)(F[x] + ((x > 0) ? C[x - 1] : 0));
-        wB[x] = (uint32_t)(B[x] + C[x]);
+        wF[x] = (s32Pf[c[x + 1]] - s32Pf[c[x]]) + ((x > 0) ? s32C[c[x] - 1] : 0u);
+        wB[x] = (s32Pb[c[x + 1]] - s32Pb[c[x]]) + ((x < P - 1) ? s32C[c[x + 1] - 1] : 0u);
       }
-      const uint32_t t32 = sim_fast_bits<P>(m, wF, wB, A.S, A.CR, br);
+      const uint32_t t32 = sim_bits16<P>(m, wF, wB, A.S, A.CR, br, one);
+      const int ri = code & 3;  // the start's result goes to index 0
       if (t32 >= A.S) {
-        s_aband[s] = 1;
+        s_aband[w][sl] = 1;
       } else {
-        s_chT[s][idx] = t32;
-        s_chM[s][idx] = (int8_t)(m <= 127 ? backtrack_master_bl<P, 8>(m, br)
-                                          : backtrack_master_bl<P, 16>(m, br));
+        s_chT[w][sl][ri] = t32;
+        s_chM[w][sl][ri] = (int8_t)backtrack_rows<P, 8>(m, br);
       }
-      atomicSub(&s_pend[s], 1);
+      atomicSub(&s_pend[w][sl], 1);
     }
-    __syncthreads();
-    if (tid == 0) s_head = head + nj;
+    head[0] += nj0;
+    head[1] += nj1;
+    __syncwarp();
   }
   if (A.sims) {
     unsigned long long sm = my_sims;
 #pragma unroll
     for (int o = 16; o >= 1; o >>= 1) sm += __shfl_xor_sync(0xffffffffu, sm, o);
-    if ((tid & 31) == 0 && sm) atomicAdd(A.sims, sm);
+    if (lane == 0 && sm) atomicAdd(A.sims, sm);
   }
   block_min_atomic(my_key, A.key);
 }
@@ -2616,8 +2672,7 @@ cudaError_t launch_minlb(const DevTables& t, int p, int m, int K, int16_t* arg, 
 template <int P>
 static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   EvalArgs A = A0;
-  const size_t base = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
-                      (A.fastS ? eval_fast_smem(A.t.n) : 0);
+  const size_t base = (tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15);
   int threads = 128;
   size_t smem = base;
   if (A.master) {
@@ -2651,16 +2706,43 @@ static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   return cudaGetLastError();
 }
 
+template <int P>
+static cudaError_t eval_fast_P(const EvalArgs& A, cudaStream_t s, int* launches) {
+  const int threads = 128;
+  const size_t smem = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
+                      eval_fast_smem(A.t.n) +
+                      (A.master ? (size_t)bits16_words(A.m, P) * 2 * threads : 0);
+  cudaError_t e = set_smem((const void*)k_eval_fast<P>, smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0, dev = 0;
+  cudaGetDevice(&dev);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval_fast<P>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  int64_t blocks = (A.count + threads - 1) / threads;
+  const int64_t wave = (int64_t)num_sms(dev) * occ;
+  if (blocks > wave) blocks = wave;
+  if (blocks > 0) {
+    k_eval_fast<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+    if (launches) ++*launches;
+  }
+  return cudaGetLastError();
+}
+
 cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, const int32_t* cuts,
                         int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
                         int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches,
                         int s_const, int s_iota, uint32_t fastS, int fastCR, int div1) {
   EvalArgs A{t, p, m, cuts, cuts_stride, kptr, k_const, k_iota, count, time_ns, master, nullptr,
-             s_const, s_iota, fastS, fastCR < 1 ? 1 : fastCR, div1, nullptr, nullptr};
+             s_const, s_iota, fastS, fastCR < 1 ? 1 : fastCR, div1, nullptr, nullptr, 1u};
   uint32_t* gbits = nullptr;
   unsigned int* redo = nullptr;
   if (fastS && count >= (1ll << 32)) fastS = A.fastS = 0;  // redo indices are 32-bit
+  // the fast kernel covers p == P in {2, 4, 8, 16} (exact-P templates), m >= p, and the
+  // north-star slicing form (s = 1); everything else is the generic kernel's
+  if (!(pick_P(p) == p && p >= 2 && p <= 16 && m >= p && s_const == 1 && !s_iota))
+    fastS = A.fastS = 0;
   if (fastS) {
     cudaError_t e = cudaMallocFromPoolAsync((void**)&redo, 4 * ((size_t)count + 1), pool, s);
     if (e != cudaSuccess) return e;
@@ -2672,8 +2754,7 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
     const int rows = m + min(p - 1, m);
     const int P = pick_P(p);
     const size_t per = (size_t)rows * (P <= 16 ? 1 : 2) * 4;
-    const size_t base = ((tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15)) +
-                        (fastS ? eval_fast_smem(t.n) : 0);
+    const size_t base = (tables_smem_bytes(t.npad, t.n) + 15) & ~size_t(15);
     if (per * 32 > 200 * 1024 - base) {
       cudaError_t e = cudaMallocFromPoolAsync((void**)&gbits, per * (size_t)count + 16, pool, s);
       if (e != cudaSuccess) return e;
@@ -2690,10 +2771,20 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
       default: return eval_P<32>(X, s, launches);
     }
   };
-  e = run(A);
+  if (redo) {
+    switch (p) {
+      case 2: e = eval_fast_P<2>(A, s, launches); break;
+      case 4: e = eval_fast_P<4>(A, s, launches); break;
+      case 8: e = eval_fast_P<8>(A, s, launches); break;
+      default: e = eval_fast_P<16>(A, s, launches); break;
+    }
+  } else {
+    e = run(A);
+  }
   if (e == cudaSuccess && redo) {
-    // exact int64 pass over the candidates that reached the u32 bound (one wave; it
-    // reads the count on the device and exits at once when the list is empty)
+    // exact int64 pass over the candidates the fast kernel listed (saturated ones, and
+    // T + master at k > 1); one wave, it reads the count on the device and exits at
+    // once when the list is empty
     EvalArgs X = A;
     X.fastS = 0;
     X.redo = nullptr;
@@ -2874,11 +2965,11 @@ static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev, uint64_t n
 template <int P>
 static cudaError_t heur_pool_P(const HeurArgs& A, cudaStream_t s, int dev, uint64_t nwork) {
   const int threads = hpool::NT;
-  const int rows = A.m + min(A.p - 1, A.m);
   const size_t narg = (size_t)(A.t.n + 1) * (A.p + 1);
   const size_t base = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
-                      ((narg + 7) & ~size_t(7)) * 2 + 32 * 4;
-  const size_t smem = base + (size_t)rows * 4 * threads;
+                      ((narg + 7) & ~size_t(7)) * 2 + 32 * 4 +
+                      (size_t)(2 * (A.t.n + 1) + ((A.t.n + 3) & ~3)) * 4;
+  const size_t smem = base + (size_t)bits16_words(A.m, P) * 2 * threads;
   // the static slot state plus the dynamic part can pass 48 KB while the dynamic part
   // alone does not, so the attribute is always set
   cudaError_t e = cudaFuncSetAttribute((const void*)k_heur_pool<P>,
@@ -2888,8 +2979,12 @@ static cudaError_t heur_pool_P(const HeurArgs& A, cudaStream_t s, int dev, uint6
   e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_heur_pool<P>, threads, smem);
   if (e != cudaSuccess) return e;
   occ = occ < 1 ? 1 : occ;
+  if (const char* ov = getenv("AP_HEUR_OCC")) {  // A/B: CTAs per SM
+    const int v = atoi(ov);
+    if (v >= 1 && v < occ) occ = v;
+  }
   uint64_t blocks = (uint64_t)num_sms(dev) * occ;
-  const uint64_t need = (nwork + hpool::NS - 1) / hpool::NS;
+  const uint64_t need = (nwork + hpool::NSW * hpool::NW - 1) / (hpool::NSW * hpool::NW);
   if (blocks > need) blocks = need;
   if (blocks < 1) blocks = 1;
   k_heur_pool<P><<<(unsigned)blocks, threads, smem, s>>>(A);
@@ -2908,6 +3003,8 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
   // pass; counter[2]: redo count; counter[3..]: redo ids (caller zeroes [0..2])
   const bool fast = fastS > 0 && pick_P(p) == p && p >= 2 && p <= 16 && m >= p && m <= 32767 &&
                     !replay_cuts;
+  // the warp pool's 8-bit master counters need 2m <= 255 (ap_master.cuh)
+  const bool pool_ok = m <= 127;
   HeurArgs A{t, p, m, seed, radius, r_lo, r_hi, arg, alg1_cuts, counter, key, replay_cuts, sims,
              best_out, fastS, fastCR < 1 ? 1 : fastCR, nullptr, adjust_mode};
   const uint64_t R = r_hi - r_lo;
@@ -2923,7 +3020,7 @@ cudaError_t launch_heuristic(const DevTables& t, int p, int m, uint64_t seed, in
   A.redo = counter + 2;
   cudaError_t e;
   const char* pv = getenv("AP_HEUR_POOL");  // A/B: AP_HEUR_POOL=0 runs k_heur<P, true>
-  if (adjust_mode == 0 && !(pv && pv[0] == '0')) {
+  if (adjust_mode == 0 && pool_ok && !(pv && pv[0] == '0')) {
     switch (p) {
       case 2: e = heur_pool_P<2>(A, s, dev, R); break;
       case 4: e = heur_pool_P<4>(A, s, dev, R); break;

@@ -21,8 +21,9 @@
  *  - Ownership: the plan owns its device tables.  The caller owns every buffer it
  *    passes.  Device pointers must be on the plan's device.
  *  - Synchronisation: calls that write device outputs are asynchronous and
- *    stream-ordered on `stream` (ap_eval_batch, ap_search_*), except that
- *    ap_search_* synchronise once on `stream` to read the reference time T_ref.
+ *    stream-ordered on `stream` (ap_eval_batch, ap_search_*): nothing in them waits
+ *    for the device (the reference time T_ref and everything derived from it are
+ *    computed and consumed on the device), so they can be captured in a CUDA graph.
  *    Calls with host outputs block until they are ready.
  *  - Errors: every call returns an ap_status.  The message of the most recent
  *    failure on the calling thread is available from ap_last_error().  On error
@@ -45,6 +46,13 @@ typedef struct CUstream_st* ap_stream_t; /* == cudaStream_t; NULL = legacy defau
 #define AP_MAX_P 32   /* pipeline stages  */
 #define AP_MAX_K 16   /* slice pieces of micro-batch 0 */
 #define AP_MAX_N 512  /* sub-layers       */
+
+/* Packed exhaustive key written when T_ref << rb | index does not fit in 63 bits (the
+ * test needs T_ref, known only on the device, so it cannot be a return status of the
+ * asynchronous call).  It is the least int64, so all_reduce(MIN) over ranks keeps it
+ * and every rank switches to ap_search_exhaustive2 together; ap_decode returns
+ * AP_ERR_RANGE for it. */
+#define AP_KEY_RANGE ((int64_t)(-9223372036854775807LL - 1))
 
 typedef enum {
   AP_OK = 0,
@@ -144,10 +152,12 @@ ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t
  * the lexicographic min of (T, rank, k) ("Return the partition scheme
  * with minimum iteration time"; reading Q15), so the keys of disjoint slices on
  * different GPUs combine with one all_reduce(MIN) (BASELINE north_star).
- *   key     device int64[1] (written)
- * Synchronises `stream` once (to read T_ref), then launches asynchronously.
+ *   key     device int64[1] (written); AP_KEY_RANGE if T_ref << rb does not fit in 63
+ *           bits (then no candidate is simulated: use ap_search_exhaustive2)
+ * Asynchronous on `stream` (T_ref, S and the u32 clamp schedule are computed on the
+ * device by a one-thread kernel the sweep reads).
  * Errors: INVALID (p, m, k range, empty or out-of-range rank slice), RANGE (overflow
- * guard, or T_ref << rb does not fit in 63 bits), CUDA, NOMEM.
+ * guard), CUDA, NOMEM.
  */
 ap_status ap_search_exhaustive(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
                                int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi,
@@ -195,8 +205,7 @@ ap_status ap_search_exhaustive_mode(const ap_plan* plan, int32_t p, int32_t m, i
  * Each CTA stores its lexicographic min (T, index); one more single-CTA kernel
  * reduces those records.  Multi-GPU: all_reduce(MIN) a copy of out[0] -> T*, then
  * ap_key2_select(out, T*, idx) and all_reduce(MIN) idx; decode with ap_decode mode 2.
- * Synchronises `stream` once (to read T_ref), then launches asynchronously.
- * Errors as ap_search_exhaustive_mode, minus the key-packing RANGE.
+ * Asynchronous on `stream`.  Errors as ap_search_exhaustive_mode (no AP_KEY_RANGE).
  */
 ap_status ap_search_exhaustive2(const ap_plan* plan, int32_t p, int32_t m, int32_t k_lo,
                                 int32_t k_hi, uint64_t rank_lo, uint64_t rank_hi, int32_t mode,
@@ -248,7 +257,8 @@ ap_status ap_key2_select(const int64_t* local, const int64_t* t_star, int64_t* i
  *   master can then rise, the walk also stops when its post-adjustment scheme repeats
  *   one of its last 32 (splitmix64 hash of the cut vector); the n*p step cap holds.
  *   0 <= r_lo < r_hi <= 2^20, 0 <= radius <= 1<<20, adjust_mode in {0, 1}.
- * Synchronises `stream` once (overflow guard), then launches asynchronously.
+ * Asynchronous on `stream`.  RANGE when a simulated T could reach 2^43 (the overflow
+ * guard m*(sum f + sum b) + 2m(p-1)*max comm >= 2^43): the key holds T in 43 bits.
  */
 ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
                               int32_t radius, uint32_t r_lo, uint32_t r_hi,
@@ -269,8 +279,9 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
  *   key   device int64[1]: min over restarts of (T << 20 | r), INT64_MAX if none.
  *   0 <= r_lo < r_hi <= 2^20, 0 <= radius <= 2^20, 1 <= vmax <= 2^20; k = 1.
  * Scratch from the plan's pool: (restart groups in flight) x vmax x (2*P + 8) bytes.
- * Synchronises `stream` once (overflow guard), then launches asynchronously.
- * Errors: INVALID, RANGE (overflow guard), NOMEM (scratch), CUDA.
+ * Asynchronous on `stream`.
+ * Errors: INVALID, RANGE (overflow guard; as ap_search_heuristic, T must stay below
+ * 2^43), NOMEM (scratch), CUDA.
  */
 ap_status ap_search_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_t seed,
                               int32_t radius, uint32_t r_lo, uint32_t r_hi, int32_t vmax,
@@ -385,7 +396,8 @@ ap_status ap_min_lower_bound(const ap_plan* plan, int32_t p, int32_t m, int32_t 
                              int32_t* cuts);
 
 /* Details of the last ap_search_exhaustive launch on this thread (for benches):
- * which sweep variant ran and its grid. */
+ * which sweep variant ran and its grid.  t_ref, fast_u32 and the clamp fields are
+ * computed on the device; this call waits for the last search to read them. */
 typedef struct {
   int32_t fast_u32;        /* 1: exact u32 saturating sweep, 0: int64 sweep        */
   int32_t exact_p;         /* 1: kernel specialised for this p, 0: generic        */

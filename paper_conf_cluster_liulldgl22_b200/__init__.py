@@ -23,6 +23,7 @@ AP_MAX_P = 32
 AP_MAX_K = 16
 AP_MAX_N = 512
 INT64_MAX = (1 << 63) - 1
+AP_KEY_RANGE = -(1 << 63)  # include/ap.h: packed exhaustive key that does not fit
 AP_OK, AP_ERR_INVALID, AP_ERR_RANGE, AP_ERR_CUDA, AP_ERR_NOMEM, AP_ERR_CAPACITY = range(6)
 
 _STATUS = {0: "AP_OK", 1: "AP_ERR_INVALID", 2: "AP_ERR_RANGE", 3: "AP_ERR_CUDA",

@@ -51,6 +51,21 @@ struct KernelTimer {
   bool truncated_valid = false;  // the last search was ap_search_reachable
   unsigned long long* d_sims = nullptr;
   int d_sims_dev = -1;
+  // SweepDev of the last exhaustive search (written by k_sweep_prep on the device);
+  // ap_last_launch reads it once the search has completed
+  apk::SweepDev* d_sweep = nullptr;
+  int d_sweep_dev = -1;
+  bool sweep_pending = false;
+  cudaError_t sweep_buffer(int device, apk::SweepDev** out) {
+    if (d_sweep_dev != device) {
+      d_sweep = nullptr;  // (a buffer of another device is leaked; one per thread/device switch)
+      cudaError_t e = cudaMalloc((void**)&d_sweep, sizeof(apk::SweepDev));
+      if (e != cudaSuccess) return e;
+      d_sweep_dev = device;
+    }
+    *out = d_sweep;
+    return cudaSuccess;
+  }
   cudaError_t sims_buffer(int device, unsigned long long** out) {
     if (d_sims_dev != device) {
       d_sims = nullptr;  // (a buffer of another device is leaked; one per thread/device switch)
@@ -233,6 +248,20 @@ const char* ap_last_error(void) { return g_err.c_str(); }
 const char* ap_version(void) { return "autopipe-b200 0.1 (sm_100a)"; }
 
 void ap_last_launch(ap_launch_info* info) {
+  if (g_timer.sweep_pending && g_timer.d_sweep) {
+    // the T_ref-dependent fields come from the device (k_sweep_prep): wait for the
+    // search, then read them once
+    apk::SweepDev d{};
+    if (cudaEventSynchronize(g_timer.ev[1]) == cudaSuccess &&
+        cudaMemcpy(&d, g_timer.d_sweep, sizeof(d), cudaMemcpyDeviceToHost) == cudaSuccess) {
+      g_last.t_ref = d.tref;
+      g_last.fast_u32 = g_last.fast_u32 && d.u32;
+      g_last.clamp_rows = g_last.fast_u32 ? d.clamp_rows : 0;
+      g_last.clamp_first = g_last.fast_u32 ? d.clamp_first : 0;
+      g_last.clamp_final = g_last.fast_u32 ? d.clamp_final : 0;
+    }
+    g_timer.sweep_pending = false;
+  }
   if (info) *info = g_last;
 }
 
@@ -447,6 +476,16 @@ ap_status check_pm(const ap_plan* plan, int p, int m) {
   return AP_OK;
 }
 
+// Restart keys pack T << 20 | r (T < 2^43): the overflow guard's bound on any T must fit.
+ap_status check_key43(const ap_plan* plan, int p, int m) {
+  const unsigned __int128 tot = (unsigned __int128)m * (uint64_t)(plan->sum_f + plan->sum_b) +
+                                (unsigned __int128)2 * m * (p - 1) * (uint64_t)plan->max_comm;
+  if (tot >= ((unsigned __int128)1 << 43))
+    return fail(AP_ERR_RANGE, "restart key packing: a T up to the overflow guard's bound needs "
+                "more than 43 bits");
+  return AP_OK;
+}
+
 cudaStream_t S_(ap_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
 
 }  // namespace
@@ -633,86 +672,59 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   int launches = 1;
   AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 1, nk,
                            d_tref, nullptr, s, &launches));
-  int64_t trefs[AP_MAX_K];
-  int32_t a1h[32] = {0};
-  AP_CUDA(cudaMemcpyAsync(trefs, d_tref, 8 * (size_t)nk, cudaMemcpyDeviceToHost, s));
-  if (mem && p > 1) AP_CUDA(cudaMemcpyAsync(a1h, d_a1, 4 * (size_t)(p - 1), cudaMemcpyDeviceToHost, s));
-  AP_CUDA(cudaStreamSynchronize(s));
-  int64_t tref = trefs[0];
-  for (int i = 0; i < nk; ++i) {
-    if (trefs[i] < 0) return fail(AP_ERR_CUDA, "T_ref evaluation failed");
-    if (trefs[i] < tref) tref = trefs[i];
-  }
-  if (mem && !plan->feasible(p, m, a1h)) {
-    // the Alg.-1 partition does not fit: no attained feasible T to bound the search
-    // with, so every candidate stays (S = the overflow guard's bound on any T)
-    const unsigned __int128 tot = (unsigned __int128)m * (uint64_t)(plan->sum_f + plan->sum_b) +
-                                  (unsigned __int128)2 * m * (p - 1) * (uint64_t)plan->max_comm;
-    tref = (int64_t)tot;
-  }
-  if (t_bound < tref) tref = t_bound;  // caller's attained bound (ap_search_exhaustive_bounded)
-  if (key && (rb >= 63 || (uint64_t)tref >= ((1ull << (63 - rb)) - 1)))
-    return fail(AP_ERR_RANGE, "key packing: T_ref=%lld needs %d bits + %d rank bits > 63",
-                (long long)tref, bitlen((unsigned __int128)tref), rb);
-  // exact u32 saturating fast path: S = T_ref + 1.  Between two
-  // clamps every running value grows by at most W_row per row of the sweep, so with
-  // R_allow = floor((2^32-1-S)/W_row) rows per clamp segment nothing wraps.  The
-  // segments are: rows 0..p-1 (pieces + warm-up + first 1F1B row), blocks of
-  // clamp_rows steady rows, and the p-1 cool-down rows.
-  //
-  // Schedule (clamp_first / clamp_rows / clamp_final): A0 = rows a value may grow from 0 (the
-  // first segment: p warm-up rows + clamp_first steady rows), r_allow = rows from S
-  // (every later segment; the last one plus the p cool-down rows).  With C4 the whole
-  // schedule is ONE clamp.
-  const uint64_t S = (uint64_t)tref + 1;
+  // Everything that depends on T_ref -- S = T_ref + 1, the u32 choice, its clamp
+  // schedule, the key-packing test -- is computed on the device (k_sweep_prep) and read
+  // by the sweep kernels: no host synchronisation inside the search.
+  // The host only decides what cannot depend on T_ref: which kernels exist for this
+  // (p, m, mode) and whether a u32 sweep is possible at all (S >= 1).
   const unsigned __int128 wrow = (unsigned __int128)(plan->sum_f + plan->sum_b) +
                                  (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
   const unsigned __int128 lim = ((unsigned __int128)1 << 32) - 1;
-  const int64_t a0 = (int64_t)(lim / wrow);
-  const int64_t r_allow = (S >= lim) ? -1 : (int64_t)((lim - S) / wrow);
-  // (p + 1: after a clamp the offset-form sweep's conversion back to finishes can sit
-  // one row's growth above S before the p cool-down rows)
-  int want_u32 = r_allow >= (int64_t)p + 1;
-  int clamp_first = 0, clamp_rows = 1, clamp_final = 1;
-  if (want_u32) {
-    auto whole = [](int64_t r) { return r >= 8 ? (r & ~int64_t(7)) : (r >= 4 ? (r & ~int64_t(3)) : r); };
-    const int64_t steady = m - p;
-    if (steady + 2 * (int64_t)p <= a0) {
-      clamp_first = (int)steady + 1;  // no clamp at all
-      clamp_rows = m;
-      clamp_final = 0;
-    } else {
-      int64_t s1 = a0 - p;
-      if (s1 >= 1) s1 = whole(s1 < steady ? s1 : steady);
-      else s1 = 0;  // clamp right after the warm-up
-      clamp_first = (int)s1;
-      const int64_t L = steady - s1;
-      int64_t every = L < r_allow ? L : r_allow;
-      every = every >= 1 ? whole(every) : 1;
-      clamp_rows = (int)every;
-      if (L == 0) {
-        clamp_final = 1;
-      } else {
-        const int64_t last = L - every * ((L - 1) / every);
-        // + 1: the offset-form sweep converts N back to finishes (FF = N + c) before the
-        // p cool-down rows, one more row of growth
-        clamp_final = (last + p + 1 > r_allow) ? 1 : 0;
-      }
-    }
-  }
   // test/bench overrides: AP_SWEEP=int64 disables the u32 path, AP_SWEEP=generic
   // also the p-specialised kernel (both remain exact)
   const char* ov = getenv("AP_SWEEP");
   int force_generic = 0;
-  if (ov && strcmp(ov, "int64") == 0) want_u32 = 0;
-  if (ov && strcmp(ov, "generic") == 0) { want_u32 = 0; force_generic = 1; }
+  bool allow_u32 = !mem;
+  if (ov && strcmp(ov, "int64") == 0) allow_u32 = false;
+  if (ov && strcmp(ov, "generic") == 0) {
+    allow_u32 = false;
+    force_generic = 1;
+  }
+  if (mem) force_generic = 1;  // memory mode: the generic exact kernel with the filter
+  const bool exact = apk::sweep_has_exact(p, m, mem ? AP_SEARCH_FULL : mode, force_generic, mem);
+  // u32 needs r_allow = floor((2^32-1-S)/W) >= p + 1 for some S >= 1
+  const int try_u32 = (allow_u32 && exact && (unsigned __int128)(p + 2) * wrow < lim) ? 1 : 0;
+  apk::SweepDev* d_sweep = nullptr;
+  AP_CUDA(g_timer.sweep_buffer(plan->device, &d_sweep));
+  if (key) AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), nullptr, s));
+  {
+    apk::PrepArgs pa{};
+    pa.trefs = reinterpret_cast<const long long*>(d_tref);
+    pa.nk = nk;
+    pa.p = p;
+    pa.m = m;
+    pa.rb = rb;
+    pa.try_u32 = try_u32;
+    pa.wrow = (unsigned long long)wrow;
+    pa.t_bound = t_bound;
+    pa.key = reinterpret_cast<unsigned long long*>(key);
+    pa.n = plan->n;
+    if (mem) {
+      // the overflow guard's bound on any T (every candidate stays) if Alg. 1's
+      // partition does not fit
+      const unsigned __int128 tot = (unsigned __int128)m * (uint64_t)(plan->sum_f + plan->sum_b) +
+                                    (unsigned __int128)2 * m * (p - 1) * (uint64_t)plan->max_comm;
+      pa.a1 = d_a1;
+      pa.mem = plan->d_mem;
+      pa.mem_cap = plan->mem_cap;
+      pa.mem_tot = (long long)tot;
+    }
+    AP_CUDA(apk::launch_sweep_prep(pa, d_sweep, s));
+    ++launches;
+  }
   apk::SweepPlan sp{};
   unsigned long long* rec = nullptr;
-  if (key) {
-    AP_CUDA(apk::launch_init_key(reinterpret_cast<unsigned long long*>(key), nullptr, s));
-  } else {
-    AP_CUDA(sc.get((void**)&rec, 16 * (size_t)apk::sweep_max_blocks(plan->device)));
-  }
+  if (!key) AP_CUDA(sc.get((void**)&rec, 16 * (size_t)apk::sweep_max_blocks(plan->device)));
   // warp-dynamic work cursor for the p-specialised sweep;
   // AP_SWEEP_SCHED=static keeps the one-chunk-per-thread split (A/B measurements)
   unsigned long long* ctr = nullptr;
@@ -724,33 +736,27 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   const char* dv = getenv("AP_DIV1");
   const int div1 = (plan->sum_f < (1ll << 28) && plan->max_comm < (1ll << 28) &&
                     !(dv && dv[0] == '0')) ? 1 : 0;
-  if (mem) {
-    want_u32 = 0;  // memory mode: the generic exact kernel with the feasibility filter
-    force_generic = 1;
-  }
-  AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, S, rb, want_u32,
-                            clamp_rows, force_generic, mem ? AP_SEARCH_FULL : mode,
+  AP_CUDA(apk::launch_sweep(plan->dev(), p, m, k_lo, k_hi, rank_lo, rank_hi, d_sweep, rb, try_u32,
+                            force_generic, mem ? AP_SEARCH_FULL : mode,
                             reinterpret_cast<unsigned long long*>(key), s, &sp, rec,
-                            mem ? plan->d_mem : nullptr, plan->mem_cap, ctr, clamp_first,
-                            clamp_final, div1));
+                            mem ? plan->d_mem : nullptr, plan->mem_cap, ctr, div1));
+  launches += (exact && try_u32) ? 2 : 1;
   if (rec) {
     AP_CUDA(apk::launch_reduce2(rec, sp.blocks, reinterpret_cast<long long*>(out2), s));
     ++launches;
   }
   AP_CUDA(g_timer.record(1, s, plan->device));
   g_timer.sims_on_device = false;
+  g_timer.sweep_pending = true;
   g_timer.host_sims = (rank_hi - rank_lo) * (uint64_t)(k_hi - k_lo + 1);
-  launches += 2;
+  if (key) ++launches;  // k_init_key
   info.fast_u32 = sp.fast_u32;
   info.exact_p = sp.exact_p;
   info.blocks = sp.blocks;
   info.threads = sp.threads;
   info.chunk = sp.chunk;
-  info.t_ref = tref;
+  info.t_ref = -1;       // device values, filled in by ap_last_launch
   info.rank_bits = rb;
-  info.clamp_rows = sp.fast_u32 ? clamp_rows : 0;
-  info.clamp_first = sp.fast_u32 ? clamp_first : 0;
-  info.clamp_final = sp.fast_u32 ? clamp_final : 0;
   info.launches = launches;
   g_last = info;
   return AP_OK;
@@ -834,6 +840,8 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   if (!key) return fail(AP_ERR_INVALID, "key is NULL");
   if (adjust_mode != 0 && adjust_mode != 1)
     return fail(AP_ERR_INVALID, "adjust_mode %d (0 none, 1 Eq. (1))", adjust_mode);
+  st = check_key43(plan, p, m);
+  if (st != AP_OK) return st;
   if (r_lo >= r_hi || r_hi > (1u << 20)) return fail(AP_ERR_INVALID, "restart range [%u, %u)", r_lo, r_hi);
   if (radius < 0 || radius > (1 << 20)) return fail(AP_ERR_INVALID, "radius %d", radius);
   cudaStream_t s = S_(stream);
@@ -853,10 +861,11 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   const size_t need = (size_t)(r_hi - r_lo) * (size_t)(p > 1 ? p - 1 : 1) * 2;
   g_hcache.valid = false;
   if (g_hcache.dev != plan->device || g_hcache.cap < need) {
-    if (g_hcache.d_best && g_hcache.dev == plan->device) cudaFree(g_hcache.d_best);
+    // stream-ordered (no device-wide synchronisation inside the search)
+    if (g_hcache.d_best && g_hcache.dev == plan->device) cudaFreeAsync(g_hcache.d_best, s);
     g_hcache.d_best = nullptr;
     g_hcache.cap = 0;
-    AP_CUDA(cudaMalloc((void**)&g_hcache.d_best, need));
+    AP_CUDA(cudaMallocFromPoolAsync((void**)&g_hcache.d_best, need, plan->pool, s));
     g_hcache.cap = need;
     g_hcache.dev = plan->device;
   }
@@ -891,6 +900,8 @@ ap_status ap_search_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_
   ap_status st = check_pm(plan, p, m);
   if (st != AP_OK) return st;
   if (!key) return fail(AP_ERR_INVALID, "key is NULL");
+  st = check_key43(plan, p, m);
+  if (st != AP_OK) return st;
   if (r_lo >= r_hi || r_hi > (1u << 20)) return fail(AP_ERR_INVALID, "restart range [%u, %u)", r_lo, r_hi);
   if (radius < 0 || radius > (1 << 20)) return fail(AP_ERR_INVALID, "radius %d", radius);
   if (vmax < 1 || vmax > (1 << 20)) return fail(AP_ERR_INVALID, "vmax %d outside [1, 2^20]", vmax);
@@ -1024,6 +1035,9 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
   ap_status st = check_pm(plan, p, m);
   if (st != AP_OK) return st;
   if (!out) return fail(AP_ERR_INVALID, "out is NULL");
+  if (key == AP_KEY_RANGE)
+    return fail(AP_ERR_RANGE, "key packing: T_ref << rank bits does not fit in 63 bits "
+                "(use ap_search_exhaustive2)");
   if (key == INT64_MAX || key < 0) return fail(AP_ERR_INVALID, "empty key (no candidate found)");
   memset(out, 0, sizeof *out);
   out->p = p;

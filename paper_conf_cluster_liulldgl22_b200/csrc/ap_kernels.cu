@@ -361,7 +361,84 @@ struct SweepArgs {
   int64_t mem_cap;
   unsigned long long* ctr;  // non-null: warp-dynamic work cursor (zeroed), chunk = ranks/lane/unit
   int div1;                 // u32: all stage computes / comms < 2^28, one-umulhi floor(v/k)
+  const SweepDev* dp;       // S and the clamp schedule (k_sweep_prep, stream-ordered)
+  int is_u32;               // this launch is the u32 variant
 };
+
+// k_sweep_prep: T_ref -> S, u32 choice and clamp schedule, on the device.
+// Same arithmetic as the host had: T_ref = min_k T(Alg.-1 partition, k) (or the memory
+// mode's fallback), capped by the caller's bound; S = T_ref + 1; with W = wrow the
+// growth per row, A0 = floor((2^32-1)/W) rows from 0 and R = floor((2^32-1-S)/W) rows
+// from a clamp at S; u32 iff R >= p + 1.
+__global__ void k_sweep_prep(PrepArgs a, SweepDev* out) {
+  long long tref = a.trefs[0];
+  for (int i = 1; i < a.nk; ++i) tref = a.trefs[i] < tref ? a.trefs[i] : tref;
+  if (a.mem) {
+    // reading R-N4: the Alg.-1 partition must fit, else every candidate stays
+    bool fits = true;
+    const int n = a.n, p = a.p;
+    int lo = 0;
+    for (int x = 0; x < p; ++x) {
+      const int hi = (x < p - 1) ? a.a1[x] : n;
+      const long long inflight = (p - x < a.m) ? p - x : a.m;
+      const long long need = (a.mem[hi] - a.mem[lo]) + inflight * (a.mem[n + 1 + hi] - a.mem[n + 1 + lo]);
+      fits = fits && need <= a.mem_cap;
+      lo = hi;
+    }
+    if (!fits) tref = a.mem_tot;
+  }
+  if (a.t_bound < tref) tref = a.t_bound;
+  SweepDev d{};
+  d.tref = tref;
+  d.S = (unsigned long long)tref + 1;
+  d.skip = 0;
+  if (a.key && (a.rb >= 63 || (unsigned long long)tref >= ((1ull << (63 - a.rb)) - 1))) {
+    *a.key = 0x8000000000000000ull;  // AP_KEY_RANGE (INT64_MIN): the packed key does not fit
+    d.skip = 1;
+  }
+  const unsigned long long lim = 0xffffffffull, W = a.wrow;
+  const long long a0 = (long long)(lim / W);
+  const long long r_allow = (d.S >= lim) ? -1 : (long long)((lim - d.S) / W);
+  const int p = a.p, m = a.m;
+  int u32 = a.try_u32 && r_allow >= (long long)p + 1;
+  int clamp_first = 0, clamp_rows = 1, clamp_final = 1;
+  if (u32) {
+    auto whole = [](long long r) { return r >= 8 ? (r & ~7ll) : (r >= 4 ? (r & ~3ll) : r); };
+    const long long steady = m - p;
+    if (steady + 2 * (long long)p <= a0) {
+      clamp_first = (int)steady + 1;  // no clamp at all
+      clamp_rows = m;
+      clamp_final = 0;
+    } else {
+      long long s1 = a0 - p;
+      if (s1 >= 1) s1 = whole(s1 < steady ? s1 : steady);
+      else s1 = 0;  // clamp right after the warm-up
+      clamp_first = (int)s1;
+      const long long L = steady - s1;
+      long long every = L < r_allow ? L : r_allow;
+      every = every >= 1 ? whole(every) : 1;
+      clamp_rows = (int)every;
+      if (L == 0) {
+        clamp_final = 1;
+      } else {
+        const long long last = L - every * ((L - 1) / every);
+        // + 1: the offset-form sweep converts N back to finishes (FF = N + c) before the
+        // p cool-down rows, one more row of growth
+        clamp_final = (last + p + 1 > r_allow) ? 1 : 0;
+      }
+    }
+  }
+  d.u32 = u32;
+  d.clamp_first = clamp_first;
+  d.clamp_rows = clamp_rows < 1 ? 1 : clamp_rows;
+  d.clamp_final = clamp_final;
+  *out = d;
+}
+
+cudaError_t launch_sweep_prep(const PrepArgs& a, SweepDev* out, cudaStream_t s) {
+  k_sweep_prep<<<1, 1, 0, s>>>(a, out);
+  return cudaGetLastError();
+}
 
 AP_DEV_INLINE uint64_t binom_at(const uint64_t* binom, int a, int b) {
   return (a < 0 || b < 0 || b > a) ? 0ull : binom[a * 33 + b];
@@ -479,15 +556,22 @@ __global__ void k_key2_select(const long long* local, const long long* t_star, l
 }
 
 template <int P, typename V>
-__device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1,
-                                            const V* sPf, const V* sPb, const V* sC,
-                                            const uint32_t* s_mk, V& bestT, uint64_t& bestIdx);
+__device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1, V S,
+                                            ClampSched cs, const V* sPf, const V* sPb,
+                                            const V* sC, const uint32_t* s_mk, V& bestT,
+                                            uint64_t& bestIdx);
 
 template <int P, typename V>
 #ifndef AP_SWEEP_MINB
 #define AP_SWEEP_MINB (P <= 8 ? 3 : 2)
 #endif
 __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A) {
+  // S and the clamp schedule come from k_sweep_prep; the variant it did not pick (and
+  // every launch after a key-packing overflow) returns at once
+  const int d_u32 = A.dp->u32, d_skip = A.dp->skip;
+  if (d_skip || d_u32 != A.is_u32) return;
+  const uint64_t dS = A.dp->S;
+  const ClampSched dcs{A.dp->clamp_first, A.dp->clamp_rows, A.dp->clamp_final};
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
@@ -508,7 +592,7 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
                                  : (uint32_t)((1ull << 32) / threadIdx.x);
   __syncthreads();
 
-  const V S = (V)A.S;
+  const V S = (V)dS;
   V bestT = S;
   uint64_t bestIdx = 0;
   if (A.ctr) {
@@ -524,27 +608,26 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
       if (u * 32ull >= (span + A.chunk - 1) / A.chunk) break;
       const uint64_t r0 = A.rank_lo + (u * 32ull + (uint64_t)lane) * A.chunk;
       if (r0 < A.rank_hi)
-        sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), sPf, sPb, sC, s_mk, bestT, bestIdx);
+        sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), S, dcs, sPf, sPb, sC, s_mk, bestT, bestIdx);
     }
   } else {
     const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const uint64_t r0 = A.rank_lo + tid * A.chunk;
     if (r0 < A.rank_hi)
-      sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), sPf, sPb, sC, s_mk, bestT, bestIdx);
+      sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), S, dcs, sPf, sPb, sC, s_mk, bestT, bestIdx);
   }
   sweep_result(A, bestT < S, (uint64_t)bestT, bestIdx);
 }
 
 // Ranks [r0, r1) x k of one thread: unrank r0, then lex successors (a2-a7).
 template <int P, typename V>
-__device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1,
-                                            const V* sPf, const V* sPb, const V* sC,
-                                            const uint32_t* s_mk, V& bestT, uint64_t& bestIdx) {
+__device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1, V S,
+                                            ClampSched cs, const V* sPf, const V* sPb,
+                                            const V* sC, const uint32_t* s_mk, V& bestT,
+                                            uint64_t& bestIdx) {
   const int n = A.t.n;
   const int m = A.m, k_lo = A.k_lo, k_hi = A.k_hi;
   const uint64_t K = (uint64_t)(k_hi - k_lo + 1);
-  const V S = (V)A.S;
-  const ClampSched cs{A.clamp_first, A.clamp_rows, A.clamp_final};
   {
     // unrank r0 (reading O7 lex order)
     int c[P + 1];
@@ -739,6 +822,8 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
 // Generic exhaustive sweep: runtime p <= P, any m, exact int64.
 template <int P>
 __global__ void __launch_bounds__(128) k_sweep_generic(SweepArgs A) {
+  if (A.dp->skip) return;
+  const uint64_t dS = A.dp->S;
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
@@ -751,7 +836,7 @@ __global__ void __launch_bounds__(128) k_sweep_generic(SweepArgs A) {
     s_mem = sm;
   }
   const uint64_t K = (uint64_t)(A.k_hi - A.k_lo + 1);
-  int64_t bestT = (int64_t)A.S;
+  int64_t bestT = (int64_t)dS;
   uint64_t bestIdx = 0;
   const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const uint64_t r0 = A.rank_lo + tid * A.chunk;
@@ -821,7 +906,7 @@ __global__ void __launch_bounds__(128) k_sweep_generic(SweepArgs A) {
       }
     }
   }
-  sweep_result(A, bestT < (int64_t)A.S, (uint64_t)bestT, bestIdx);
+  sweep_result(A, bestT < (int64_t)dS, (uint64_t)bestT, bestIdx);
 }
 
 __global__ void k_init_key(unsigned long long* key) { *key = 0x7fffffffffffffffull; }
@@ -2914,22 +2999,48 @@ bool has_exact(int p) {
   return (p >= 1 && p <= 8) || p == 10 || p == 12 || p == 16;
 }
 
+bool sweep_has_exact(int p, int m, int mode, int force_generic, bool mem) {
+  return !mem && has_exact(p) && m >= p && (!force_generic || mode != 0);
+}
+
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
-                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
+                         uint64_t rank_hi, const SweepDev* dp, int rb, int try_u32,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
                          SweepPlan* sp, unsigned long long* rec, const int64_t* mem,
-                         int64_t mem_cap, unsigned long long* ctr, int clamp_first,
-                         int clamp_final, int div1) {
+                         int64_t mem_cap, unsigned long long* ctr, int div1) {
   int dev = 0;
   cudaGetDevice(&dev);
-  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, S, rb, key,
-              clamp_rows < 1 ? 1 : clamp_rows, clamp_first < 0 ? 0 : clamp_first,
-              clamp_first < 0 ? 1 : clamp_final, 1u, mode, rec, mem, mem_cap, ctr,
-              want_u32 ? div1 : 0};
-  const bool exact = !mem && has_exact(p) && m >= p && (!force_generic || mode != 0);
+  SweepArgs A{t, p, m, k_lo, k_hi, rank_lo, rank_hi, 1, 0, rb, key, 1, 0, 1, 1u, mode, rec,
+              mem, mem_cap, ctr, div1, dp, 0};
+  const bool exact = sweep_has_exact(p, m, mode, force_generic, mem != nullptr);
   sp->exact_p = exact ? 1 : 0;
-  sp->fast_u32 = (exact && want_u32) ? 1 : 0;
-  if (exact) return sweep_exact_dispatch(p, sp->fast_u32, A, s, sp, dev);
+  sp->fast_u32 = (exact && try_u32) ? 1 : 0;  // the device picks; see SweepDev::u32
+  if (rec) {
+    // records of the variant that does not run stay "empty" (all ones > any real record)
+    cudaError_t e = cudaMemsetAsync(rec, 0xff, 16 * (size_t)sweep_max_blocks(dev), s);
+    if (e != cudaSuccess) return e;
+  }
+  if (exact) {
+    int blocks = 0;
+    cudaError_t e = cudaSuccess;
+    if (try_u32) {
+      A.is_u32 = 1;
+      e = sweep_exact_dispatch(p, 1, A, s, sp, dev);
+      if (e != cudaSuccess) return e;
+      blocks = sp->blocks;
+    }
+    A.is_u32 = 0;
+    A.div1 = 0;
+    SweepPlan sp64 = *sp;
+    e = sweep_exact_dispatch(p, 0, A, s, &sp64, dev);
+    if (e != cudaSuccess) return e;
+    if (!try_u32) *sp = sp64;
+    sp->blocks = blocks > sp64.blocks ? blocks : sp64.blocks;
+    sp->fast_u32 = try_u32 ? 1 : 0;
+    sp->exact_p = 1;
+    return cudaSuccess;
+  }
+  A.div1 = 0;
   switch (pick_P(p)) {
     case 2: return sweep_generic_P<2>(A, s, sp, dev);
     case 4: return sweep_generic_P<4>(A, s, sp, dev);

@@ -32,6 +32,35 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
                         int s_const = 1, int s_iota = 0, uint32_t fastS = 0, int fastCR = 16,
                         int div1 = 0);
 
+// Sweep parameters that depend on T_ref, computed on the device by k_sweep_prep right
+// after the T_ref evaluation and read by the sweep kernels at their start, so a search
+// never waits for the host.
+struct SweepDev {
+  unsigned long long S;  // T_ref + 1 (a candidate with T >= S cannot win)
+  long long tref;
+  int u32;               // 1: the u32 saturating kernel runs, 0: the int64 one
+  int clamp_first, clamp_rows, clamp_final;  // u32 clamp schedule
+  int skip;              // 1: the packed key does not fit; *key = AP_KEY_RANGE, no sweep
+  int pad;
+};
+// Host-known inputs of k_sweep_prep.
+struct PrepArgs {
+  const long long* trefs;     // T(Alg.-1 partition, k), nk entries
+  int nk;
+  int p, m, rb;
+  int try_u32;                // the u32 kernel exists for this search (exact p, no override)
+  unsigned long long wrow;    // max growth of a running value per row (< 2^62)
+  long long t_bound;          // caller's attained bound (INT64_MAX: none)
+  unsigned long long* key;    // packed-key searches: written with AP_KEY_RANGE on overflow
+  // memory mode: the Alg.-1 partition must fit, else T_ref = mem_tot
+  const int32_t* a1;          // Alg.-1 cut vector (device)
+  const int64_t* mem;         // [2][n+1] static / stash prefix sums, or null
+  int64_t mem_cap;
+  long long mem_tot;
+  int n;
+};
+cudaError_t launch_sweep_prep(const PrepArgs& a, SweepDev* out, cudaStream_t s);
+
 struct SweepPlan {
   int fast_u32;   // exact u32 saturating sweep
   int exact_p;    // kernel specialised to this p
@@ -46,13 +75,18 @@ struct SweepPlan {
 // u32 clamp schedule: clamp_first steady rows before the first clamp (-1: legacy =
 // clamp after the warm-up and at the end), then every clamp_rows, clamp_final = one
 // more clamp at the end of the steady rows.
+// The sweep reads S and the clamp schedule from `dp` (k_sweep_prep).  With try_u32 the
+// u32 and the int64 kernels are both launched and each returns at once unless dp->u32
+// selects it; plan_out->blocks is the larger grid (records of two-phase searches are
+// preset to "empty" so the idle variant's slots are neutral).
 cudaError_t launch_sweep(const DevTables& t, int p, int m, int k_lo, int k_hi, uint64_t rank_lo,
-                         uint64_t rank_hi, uint64_t S, int rb, int want_u32, int clamp_rows,
+                         uint64_t rank_hi, const SweepDev* dp, int rb, int try_u32,
                          int force_generic, int mode, unsigned long long* key, cudaStream_t s,
                          SweepPlan* plan_out, unsigned long long* rec = nullptr,
                          const int64_t* mem = nullptr, int64_t mem_cap = 0,
-                         unsigned long long* ctr = nullptr, int clamp_first = -1,
-                         int clamp_final = 1, int div1 = 0);
+                         unsigned long long* ctr = nullptr, int div1 = 0);
+// The host-side test whether the p-specialised kernel serves this (p, m, mode).
+bool sweep_has_exact(int p, int m, int mode, int force_generic, bool mem);
 
 // Two-phase reduction (NEXT N3).  With `rec` (u64[2 * sweep_max_blocks(dev)]) passed
 // to launch_sweep, each CTA stores its lexicographic min (T, index) there instead of

@@ -15,7 +15,7 @@ from typing import Optional
 
 import torch
 
-from . import (AP_ERR_RANGE, AP_SEARCH_MEMORY, INT64_MAX, APError, Plan, ap_count, ap_decode,
+from . import (AP_ERR_RANGE, AP_KEY_RANGE, AP_SEARCH_MEMORY, INT64_MAX, APError, Plan, ap_count, ap_decode,
                ap_key2_select, ap_search_exhaustive, ap_search_exhaustive2,
                ap_search_heuristic)
 
@@ -86,39 +86,36 @@ def search_exhaustive(plan: Plan, p: int, m: int, k_lo: int = 1, k_hi: int = 1,
                       two_phase: Optional[bool] = None, mode: int = 0) -> dict:
     """Exact argmin over all C(n-1,p-1) partitions x k in [k_lo,k_hi], sharded over
     the ranks of the default process group (if initialised).  two_phase None: the
-    packed key when it fits, else the two-phase reduction.  Every rank takes the same
-    branch: the packing test depends only on T_ref and N (global values), and when
-    N < world (an empty shard, which cannot run the test) the two-phase form is used
-    on every rank.""" 
+    packed key when it fits, else the two-phase reduction.  The packing test needs T_ref,
+    which only the device knows: a search whose key does not fit writes AP_KEY_RANGE (the
+    least int64), the MIN all-reduce hands it to every rank (an empty shard included),
+    and all ranks then run the two-phase form together."""
     rank, world, dist = _world()
     N = ap_count(plan.n, p)
     lo, hi = shard(N, rank, world)
     dev = f"cuda:{plan.device}"
     out = {"sims": (hi - lo) * (k_hi - k_lo + 1), "total_sims": N * (k_hi - k_lo + 1),
            "shard": (lo, hi), "two_phase": False}
-    if two_phase is None and N < world:
-        # some rank has an empty shard and never learns whether the packed key fits;
-        # decide without it (the same on every rank): the two-phase form always fits
-        two_phase = True
     if not two_phase:
         key = torch.empty(1, dtype=torch.int64, device=dev)
-        try:
-            if hi > lo:
-                from . import ap_search_exhaustive_mode
-                ap_search_exhaustive_mode(plan, p, m, k_lo, k_hi, lo, hi, mode, key, stream=stream)
-            else:
-                key.fill_(INT64_MAX)
-        except APError as e:
-            if two_phase is not None or e.status != AP_ERR_RANGE or "key packing" not in str(e):
-                raise
-            two_phase = True
-    if not two_phase:
+        if hi > lo:
+            from . import ap_search_exhaustive_mode
+            ap_search_exhaustive_mode(plan, p, m, k_lo, k_hi, lo, hi, mode, key, stream=stream)
+        else:
+            key.fill_(INT64_MAX)
         min_allreduce_key(key, dist, group)
         kv = int(key.item())
-        out["key"] = kv
-        if decode and kv != INT64_MAX:
-            out.update(ap_decode(plan, 0, p, m, k_lo, k_hi, key=kv))
-        return out
+        if kv == AP_KEY_RANGE:
+            # T_ref << rb does not fit (decided on the device); the MIN reduction handed
+            # the sentinel to every rank, empty shards included, so all switch together
+            if two_phase is not None:
+                raise APError(AP_ERR_RANGE, "key packing: the packed key does not fit")
+            two_phase = True
+        else:
+            out["key"] = kv
+            if decode and kv != INT64_MAX:
+                out.update(ap_decode(plan, 0, p, m, k_lo, k_hi, key=kv))
+            return out
     local = torch.empty(2, dtype=torch.int64, device=dev)
     if hi > lo:
         ap_search_exhaustive2(plan, p, m, k_lo, k_hi, lo, hi, mode, local, stream=stream)

@@ -696,8 +696,13 @@ def test_two_phase_when_packed_key_does_not_fit(ap, oracle_mod):
         plan = _plan(ap, f, b, a, bw)
         p, m, k_lo, k_hi = 4, 16, 1, 4
         key = torch.empty(1, dtype=torch.int64, device="cuda")
+        # the packing test needs T_ref (device-side): the key comes back as AP_KEY_RANGE,
+        # and decoding it is the RANGE error
+        ap.ap_search_exhaustive(plan, p, m, k_lo, k_hi, 0, ap.ap_count(30, p), key)
+        torch.cuda.synchronize()
+        assert int(key.item()) == ap.AP_KEY_RANGE
         with pytest.raises(ap.APError) as ei:
-            ap.ap_search_exhaustive(plan, p, m, k_lo, k_hi, 0, ap.ap_count(30, p), key)
+            ap.ap_decode(plan, 0, p, m, k_lo, k_hi, key=int(key.item()))
         assert ei.value.status == ap.AP_ERR_RANGE
         o = M.exhaustive(p, m, k_lo, k_hi)
         assert o["T"] >= 1 << 48

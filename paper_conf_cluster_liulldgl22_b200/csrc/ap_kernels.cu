@@ -170,23 +170,35 @@ AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const 
 #pragma unroll
     for (int x = 1; x < P; ++x) FF[x] = fma_add(FF[x - 1], wF[x], one);  // FMA pipe: ALU-bound
   } else {
-    V a[P], al[P];
+    V a[P];
 #pragma unroll
     for (int x = 0; x < P; ++x) {
       const V Fx = sPf[c[x + 1]] - sPf[c[x]];
       const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
       a[x] = divk(Fx, (uint32_t)k, Mk, div1) + ((x > 0) ? divk(Cin, (uint32_t)k, Mk, div1) : V(0));
-      al[x] = wF[x] - V(k - 1) * a[x];
-      FF[x] = 0;
     }
-    for (int q = 0; q < k - 1; ++q) {
-      FF[0] = O::ad(FF[0], a[0], one);
+    // Offset form: piece q's finish FF_q[x] = max(FF_q[x-1],
+    // FF_{q-1}[x]) + a_x.  With s_x = a_0 + .. + a_x (= FF_0[x]) and E_q = FF_q - s,
+    //   E_q[x] = max(E_{q-1}[x] + a_x, E_q[x-1]),  E_q[0] = q a_0,  E_0 = 0,
+    // one fused add+max per op; E >= 0 because FF_q >= FF_0.  The last piece (weights
+    // al_x = wF_x - (k-1) a_x) reads FF_{k-2}[x] = E[x] + s_x.
+    V E[P];
 #pragma unroll
-      for (int x = 1; x < P; ++x) FF[x] = O::ad(O::mx(FF[x - 1], FF[x]), a[x], one);
+    for (int x = 0; x < P; ++x) E[x] = 0;
+    for (int q = 1; q < k - 1; ++q) {
+      E[0] = fma_add(E[0], a[0], one);
+#pragma unroll
+      for (int x = 1; x < P; ++x) E[x] = O::amx(E[x], a[x], E[x - 1]);
     }
-    FF[0] = O::ad(FF[0], al[0], one);
+    const V km1 = V(k - 1);
+    V sxr = a[0];
+    FF[0] = fma_add(fma_add(E[0], sxr, one), wF[0] - km1 * a[0], one);
 #pragma unroll
-    for (int x = 1; x < P; ++x) FF[x] = O::ad(O::mx(FF[x - 1], FF[x]), al[x], one);
+    for (int x = 1; x < P; ++x) {
+      sxr = fma_add(sxr, a[x], one);
+      const V t = fma_add(E[x], sxr, one);  // FF_{k-2}[x]
+      FF[x] = fma_add(O::mx(FF[x - 1], t), wF[x] - km1 * a[x], one);
+    }
   }
 }
 
@@ -261,7 +273,17 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
 #pragma unroll
             for (int u = 0; u < U; ++u) nstep<P, V>(N, sw, one);
           }
-          for (; blk > 0; --blk) nstep<P, V>(N, sw, one);
+          // the remaining blk < U rows: one computed jump instead of a counted loop
+          switch (blk) {
+            case 7: if constexpr (U > 7) nstep<P, V>(N, sw, one); [[fallthrough]];
+            case 6: if constexpr (U > 6) nstep<P, V>(N, sw, one); [[fallthrough]];
+            case 5: if constexpr (U > 5) nstep<P, V>(N, sw, one); [[fallthrough]];
+            case 4: if constexpr (U > 4) nstep<P, V>(N, sw, one); [[fallthrough]];
+            case 3: nstep<P, V>(N, sw, one); [[fallthrough]];
+            case 2: nstep<P, V>(N, sw, one); [[fallthrough]];
+            case 1: nstep<P, V>(N, sw, one); [[fallthrough]];
+            default: break;
+          }
           if (rem <= 0) break;
           clamp_n<P, V>(N, S);
           blk = rem < cs.every ? rem : cs.every;
@@ -296,34 +318,29 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
   // b[x+1] = M + wB[x+1] folded into the next fused add+max.
   V b = 0;
   constexpr int TEND = REV ? P - 1 : P;
+  // Every backward of the step carries the pending weight of the one above it:
+  // b[x+1] = M + wpend, so each op is one fused add+max (VIADDMNMX) on the ALU pipe
+  // plus the adds that materialise finishes, which go to the FMA pipe.
 #pragma unroll
   for (int t = 0; t < TEND; ++t) {
     if constexpr (P == 1) {
       b = O::ad(FF[0], wB[0], one);
     } else {
-      V M = FF[P - 1];   // pending value; b[P-1] = M + wB[P-1]
-      V wpend = wB[P - 1];
+      V M = FF[P - 1];
+      V wpend = wB[P - 1];  // b[P-1] = M + wpend
 #pragma unroll
       for (int x = P - 2; x >= 0; --x) {
         if (x >= t) {
-          M = O::amx(M, wpend, FF[x]);                      // max(b[x+1], FF[x])
-          if (t < P - 1) FF[x + 1] = O::ad(M, wF[x + 1], one);  // not read again this step
-          wpend = wB[x];
-          if (x == t) {
-            L[x] = O::ad(M, wB[x], one);
-            M = L[x];
-            wpend = 0;
-          }
+          M = O::amx(M, wpend, FF[x]);  // max(b[x+1], FF[x])
+          if (t < P - 1) FF[x + 1] = fma_add(M, wF[x + 1], one);
+          if (x == t) L[x] = fma_add(M, wB[x], one);
         } else {
-          // b[x] = max(b[x+1], L[x]) + wB[x] with b[x+1] = M + wpend; wpend is 0
-          // unless stage x+1 is P-1 (its weight is still pending from the start)
-          const V bx1 = (x <= P - 3) ? M : O::ad(M, wpend, one);
-          M = O::ad(O::mx(bx1, L[x]), wB[x], one);
-          L[x] = M;
-          wpend = 0;
+          M = O::amx(M, wpend, L[x]);  // max(b[x+1], L[x]): stage x forwards no more
+          L[x] = fma_add(M, wB[x], one);
         }
+        wpend = wB[x];
       }
-      b = M;  // stage 0 is always materialised (x == t or x < t)
+      b = fma_add(M, wpend, one);  // B(0) of the row
     }
   }
   if constexpr (REV) {

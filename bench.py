@@ -50,13 +50,28 @@ def _peaks():
         return {"sm_max_mhz": 1965.0}, "fallback"
 
 
-def int_peak_ops(sm_mhz: float, sms: int = 148) -> float:
-    """Integer ALU roofline in int32 ops/s.  Per SM per clock: the alu
-    pipe retires 64 lanes (4 SMSPs x 16, rt_SMSP = 2) of instructions that each do up to
-    TWO int32 ops (VIADDMNMX = add + max, IADD3 = two adds), and the fmaheavy pipe 64
-    lanes of IMAD (one add).  Issue (1 warp-instruction/clk/SMSP = 128 lanes) is not
-    binding beyond that.  Peak = 148 x (64*2 + 64*1) = 192 int32 ops/clk/SM."""
-    return sms * 192 * sm_mhz * 1e6
+INTPEAK = os.path.join(ROOT, "profiles", "r02_intpeak.json")
+
+
+def int_peak(sm_mhz: float, sms: int = 148):
+    """Integer roofline in int32 ops/s.  The max-plus work runs on two
+    pipes: the ALU pipe, whose VIADDMNMX does two int32 ops (add + max), and the FMA pipe,
+    whose IMAD does one add.  The denominator is MEASURED on the B200 by the builder's
+    microbenchmark (tools/microbench/intpeak.cu, committed result profiles/r02_intpeak.json):
+    a 1:1 VIADDMNMX:IMAD mix with 8 independent chains per thread reaches 185.7 int32
+    ops/clk/SM (0.967 warp-instructions/clk/SMSP; the two single-pipe rates are 0.499
+    each).  Scaled to the clock measured during the bench's timed region.
+    Returns (ops/s, ops/clk/SM, source string)."""
+    try:
+        with open(INTPEAK) as fh:
+            d = json.load(fh)
+        per = float(d["modes"]["mix11"]["int32_ops_per_clk_per_sm"])
+        src = ("measured (builder microbench tools/microbench/intpeak.cu, 1:1 VIADDMNMX:IMAD, "
+               f"profiles/r02_intpeak.json: {per:.1f} int32 ops/clk/SM)")
+    except Exception:
+        per = 192.0
+        src = "fallback: 64 ALU lanes x 2 ops + 64 FMA lanes x 1 op per clk per SM (guide pipe rates)"
+    return sms * per * sm_mhz * 1e6, per, src
 
 
 NCU_PROFILE = os.path.join(ROOT, "profiles", "ncu_sweep_c4.json")
@@ -154,33 +169,91 @@ def cpu_model():
 
 
 # ----------------------------------------------------------------------------- oracle
-def oracle_rate(wl, budget_s: float = 24.0, threads: int = 0):
-    """The oracle as it stands (plain C DAG simulator, brute force in lex order) on
-    the host cores, on a bounded sample of the workload: contiguous rank windows
-    starting at evenly spaced ranks, all k each.  Returns sims/s."""
+def _oracle_window_rate(M, wl, N, budget_s, threads, nwin):
+    """One time-boxed oracle run: `nwin` contiguous lex-rank windows starting at evenly
+    spaced ranks; `threads` host threads visit their windows round-robin, simulating one
+    batch of ~256 (partition, k) pairs per visit (the C oracle releases the GIL), until
+    `budget_s` of wall time has passed.  Each thread calibrates itself: it stops on its own
+    clock, so a slow core does not hold the others."""
+    from concurrent.futures import ThreadPoolExecutor
+    K = wl.k_hi - wl.k_lo + 1
+    batch = max(1, 256 // K)
+    starts = [N * i // nwin for i in range(nwin)]
+    pos = list(starts)
+    ends = [starts[i + 1] if i + 1 < nwin else N for i in range(nwin)]
+    t0 = time.perf_counter()
+
+    def worker(t):
+        sims = 0
+        mine = list(range(t, nwin, threads))
+        while time.perf_counter() - t0 < budget_s:
+            progressed = False
+            for w in mine:
+                if pos[w] >= ends[w]:
+                    continue
+                hi = min(ends[w], pos[w] + batch)
+                sims += M.exhaustive(wl.p, wl.m, wl.k_lo, wl.k_hi, pos[w], hi)["sims"]
+                pos[w] = hi
+                progressed = True
+                if time.perf_counter() - t0 >= budget_s:
+                    break
+            if not progressed:
+                break
+        return sims
+
+    with ThreadPoolExecutor(threads) as ex:
+        per = list(ex.map(worker, range(threads)))
+    dt = time.perf_counter() - t0
+    return sum(per), dt
+
+
+def oracle_rate(wl, budget_s: float = 10.0, runs: int = 3, threads: int = 0):
+    """The oracle as it stands (plain C DAG simulator, brute force in lex order) on the
+    host's cores, on a bounded sample of the workload: `runs` time-boxed
+    runs of `budget_s` each over max(8, threads) evenly spaced contiguous rank windows,
+    all k; the median rate is reported with the spread of the runs."""
     import oracle
     M = oracle.Model.from_workload(wl)
     N = oracle.count(wl.n, wl.p)
     threads = threads or os.cpu_count() or 1
-    K = wl.k_hi - wl.k_lo + 1
-    # calibrate one thread on a small window
-    t0 = time.perf_counter()
-    M.exhaustive(wl.p, wl.m, wl.k_lo, wl.k_hi, 0, min(N, 64))
-    per_sim = (time.perf_counter() - t0) / (min(N, 64) * K)
-    per_thread = max(1, int(budget_s / per_sim / K / threads))
-    starts = [int(N * i / threads) for i in range(threads)]
-    from concurrent.futures import ThreadPoolExecutor
-    t0 = time.perf_counter()
-    with ThreadPoolExecutor(threads) as ex:
-        res = list(ex.map(lambda s: M.exhaustive(wl.p, wl.m, wl.k_lo, wl.k_hi, s,
-                                                 min(N, s + per_thread)), starts))
-    dt = time.perf_counter() - t0
-    sims = sum(r["sims"] for r in res)
-    return {"value": sims / dt, "unit": "sims/s", "cores": threads, "kind": "oracle",
-            "sample": f"{sims} simulations: {threads} contiguous lex-rank windows of "
-                      f"{per_thread} partitions x k in [{wl.k_lo},{wl.k_hi}] at evenly spaced "
-                      f"start ranks of the {N}-partition space ({dt:.1f} s wall)",
+    nwin = max(8, threads)
+    rates, sims_tot, wall_tot = [], 0, 0.0
+    for _ in range(runs):
+        sims, dt = _oracle_window_rate(M, wl, N, budget_s, threads, nwin)
+        rates.append(sims / dt)
+        sims_tot += sims
+        wall_tot += dt
+    med = statistics.median(rates)
+    return {"value": med, "unit": "sims/s", "cores": threads, "kind": "oracle",
+            "sims": sims_tot, "wall_s": wall_tot,
+            "runs": [round(r, 1) for r in rates],
+            "spread": (max(rates) - min(rates)) / med if med > 0 else None,
+            "sample": f"median of {runs} runs of {budget_s:.0f} s wall, each over {nwin} "
+                      f"contiguous lex-rank windows at evenly spaced start ranks of the "
+                      f"{N}-partition space, k in [{wl.k_lo},{wl.k_hi}], {threads} host threads "
+                      f"time-boxed on their own clocks ({sims_tot} simulations in {wall_tot:.1f} s)",
             "cpu": cpu_model()}
+
+
+def oracle_heuristic_rate(wl, restarts: int = 4096, runs: int = 3, threads: int = 0):
+    """The oracle's heuristic (O9) over a fixed sample of restarts [0, restarts) on the
+    host's cores: simulations/s and restarts/s, median of `runs`."""
+    import oracle
+    M = oracle.Model.from_workload(wl)
+    threads = threads or os.cpu_count() or 1
+    rates = []
+    for _ in range(runs):
+        t0 = time.perf_counter()
+        o = M.heuristic_parallel(wl.p, wl.m, wl.seed, wl.radius, 0, restarts, threads=threads)
+        dt = time.perf_counter() - t0
+        rates.append((o["sims"] / dt, restarts / dt))
+    med = statistics.median(r[0] for r in rates)
+    return {"value": med, "unit": "sims/s", "cores": threads, "kind": "oracle",
+            "restarts_per_s": statistics.median(r[1] for r in rates),
+            "runs": [round(r[0], 1) for r in rates],
+            "spread": (max(r[0] for r in rates) - min(r[0] for r in rates)) / med,
+            "sample": f"restarts [0, {restarts}) of the {wl.restarts}-restart search, "
+                      f"median of {runs} runs, {threads} host threads", "cpu": cpu_model()}
 
 
 def run_reference(args):
@@ -190,18 +263,21 @@ def run_reference(args):
     wl = synth.config(args.config)
     steps = []
     for i in range(args.warmup + args.steps):
-        r = oracle_rate(wl, budget_s=args.ref_budget)
+        r = oracle_rate(wl, budget_s=args.ref_budget, runs=1)
         if i >= args.warmup:
             steps.append(r)
     val = statistics.median(r["value"] for r in steps)
     cb = dict(steps[-1])
     cb["value"] = val
+    cb["runs"] = [round(r["value"], 1) for r in steps]
+    cb["spread"] = (max(cb["runs"]) - min(cb["runs"])) / val if val > 0 else None
+    cb["sample"] = (f"{args.steps} timed steps (after {args.warmup} warm-up), each one "
+                    f"time-boxed run: " + steps[-1]["sample"].split(", each over ", 1)[-1])
     N = synth_count(wl)
     total = N * (wl.k_hi - wl.k_lo + 1)
     out = {"impl": "reference", "metric": METRIC, "value": val, "unit": "sims/s",
            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-           "ms_per_step": 1e3 * statistics.median(
-               int(r["sample"].split()[0]) / r["value"] for r in steps),
+           "ms_per_step": 1e3 * statistics.median(r["wall_s"] for r in steps),
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
            "dtype": "int64", "data": "synthetic",
            "config": {"workload": wl.name, "n": wl.n, "p": wl.p, "m": wl.m,
@@ -311,6 +387,7 @@ def main():
     torch.cuda.synchronize()
     clocks.start()
     time.sleep(0.3)
+    launches0 = ap.ap_kernel_launches()
     wall0 = time.perf_counter()
     for i in range(args.steps):
         flush.zero_()                      # L2 flush between timed steps (untimed)
@@ -321,6 +398,7 @@ def main():
         if hi > lo:
             kern_ms.append(ap.ap_last_kernel_ms())
     torch.cuda.synchronize()
+    launches = ap.ap_kernel_launches() - launches0
     if world > 1:
         dist.barrier()
     wall = time.perf_counter() - wall0
@@ -360,13 +438,18 @@ def main():
     for mode, name in ((ap.AP_SEARCH_KFACTOR, "kfactor"), (ap.AP_SEARCH_PRUNED, "pruned")):
         kk = torch.empty(1, dtype=torch.int64, device=dev)
         def run_mode():
+            """The same time-to-optimal-plan path as step(): search, reduction, decode
+            (unrank + critical path + master) and the Slicer sweep of the winner."""
             if hi > lo:
                 ap.ap_search_exhaustive_mode(plan, wl.p, wl.m, wl.k_lo, wl.k_hi, lo, hi, mode, kk)
             else:
                 kk.fill_(ap.INT64_MAX)
             if world > 1:
                 dist.all_reduce(kk, op=dist.ReduceOp.MIN)
-            return int(kk.item())
+            kv_ = int(kk.item())
+            res_ = ap.ap_decode(plan, 0, wl.p, wl.m, wl.k_lo, wl.k_hi, key=kv_)
+            ap.ap_slice_sweep(plan, wl.p, wl.m, res_["cuts"], wl.k_hi)
+            return kv_
         for _ in range(3):
             run_mode()
         ts = []
@@ -380,6 +463,7 @@ def main():
         if world > 1:
             dist.all_reduce(tmed, op=dist.ReduceOp.MAX)
         modes[name] = {"time_to_optimal_plan_ms": float(tmed[0]),
+                       "path": "search + all_reduce + decode + Slicer sweep (as the step)",
                        "same_key_as_full": kv == int(key.item()),
                        "equivalent_candidates_per_s": total_sims / (float(tmed[0]) / 1e3)}
 
@@ -391,17 +475,21 @@ def main():
     # ------------------------------------------------------------- roofline
     k_avg_s = kern_max / max(len(kern_ms), 1)
     achieved = my_ops / k_avg_s if k_avg_s > 0 else 0.0
-    peak = int_peak_ops(sm_max, sms)
+    clk_mhz = clk.get("sm_mhz") or sm_max
+    peak, per_clk, peak_src = int_peak(clk_mhz, sms)
     roof = {"bound": "alu", "kernel": "k_sweep_exact<%d,%s>" % (wl.p, "u32" if info["fast_u32"] else "u64"),
             "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s (int32)",
             "frac": achieved / peak, "traffic": None,
+            "count": "adds + distinct maxima of the 1F1B task DAG (DESIGN.md §5.3)",
             "ops_per_launch": my_ops, "ops_per_sim_avg": my_ops / max(hi - lo, 1) / K,
             "frac_naive_count": (my_ops_naive / k_avg_s / peak) if k_avg_s > 0 else None,
+            "naive_count": "SURVEY §8d: 2 int32 ops (max + add) per max-plus op, "
+                           "2pm + (k-1)p max-plus ops per simulation",
+            "ops_per_sim_naive_avg": my_ops_naive / max(hi - lo, 1) / K,
             "kernel_ms_avg": k_avg_s * 1e3,
             "kernel_share_of_step": (kern_max / t_max) if t_max > 0 else None,
-            "peak_source": f"{sms} SMs x 192 int32 ops/clk (alu pipe 64 lanes x 2 ops fused "
-                           f"+ fmaheavy 64 lanes x 1 op) x sm_max {sm_max:.0f} MHz "
-                           f"({peak_src} MEASURED_PEAKS.json clock)",
+            "peak_source": f"{sms} SMs x {per_clk:.1f} int32 ops/clk/SM x {clk_mhz:.0f} MHz "
+                           f"(median SM clock in the timed region); {peak_src}",
             "traffic_note": "algorithmic HBM bytes per candidate = 0; traffic = ncu "
                             "dram__bytes_read+write of this kernel, one --set full capture"}
     prof = _ncu_profile()
@@ -425,7 +513,9 @@ def main():
                       "cuts": res["cuts"], "master": res["master"], "slicer_best_k": bk},
            "roofline": roof,
            "clocks": clk,
-           "gpu_launches": 7 * args.steps,
+           "gpu_launches": launches,
+           "gpu_launches_note": "libap.so kernels launched in the timed region "
+                                "(ap_kernel_launches difference), all ranks' own counts equal",
            "e2e": {"value": e2e_val, "unit": "sims/s", "h2d_bytes_per_step": tab_bytes,
                    "d2h_bytes_per_step": 8 + 8 + 140 + 8 * wl.k_hi, "steps": e2e_steps,
                    "path": "ap_plan_create(host tables) -> ap_search_exhaustive -> "
@@ -434,6 +524,10 @@ def main():
            "secondary": secondary}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = oracle_rate(wl)
+        if not args.no_secondary:
+            # same-run oracle rates beside the secondary GPU numbers
+            out["secondary"]["C3"]["cpu_baseline"] = oracle_rate(synth.config(3), budget_s=3.0)
+            out["secondary"]["C5"]["cpu_baseline"] = oracle_heuristic_rate(synth.config(5))
     if rank == 0:
         print(json.dumps(out), flush=True)
     if world > 1:

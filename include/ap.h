@@ -420,6 +420,11 @@ void ap_last_launch(ap_launch_info* info);
  * no search ran. */
 ap_status ap_last_kernel_ms(float* ms);
 
+/* Number of kernels this library has launched since it was loaded (every thread and
+ * device; a host-side counter bumped at each launch).  Benches take the difference
+ * around a timed region to state how many of the library's kernels ran in it. */
+uint64_t ap_kernel_launches(void);
+
 /* Simulations run by the last ap_search_exhaustive / ap_search_heuristic call on this
  * thread: (rank_hi-rank_lo)*(k_hi-k_lo+1) for the sweep; counted on the device for the
  * heuristic (blocks until that kernel has finished). */

@@ -75,6 +75,8 @@ def _load():
             lib.or_count.argtypes = [i32, i32]
             lib.or_rank.restype = u64
             lib.or_rank.argtypes = [i32, i32, P(i32)]
+            lib.or_unrank.restype = None
+            lib.or_unrank.argtypes = [i32, i32, u64, P(i32)]
             lib.or_exhaustive.restype = i32
             lib.or_exhaustive.argtypes = [i32, P(i64), P(i64), P(i64), i32, i32, i32, i32,
                                           u64, u64, P(i64), P(u64), P(i32), P(i32), P(u64)]
@@ -451,6 +453,12 @@ def count(n: int, p: int) -> int:
 def rank(n: int, p: int, cuts) -> int:
     c = _i32(cuts)
     return int(_load().or_rank(n, p, _p(c, C.c_int32)))
+
+
+def unrank(n: int, p: int, r: int):
+    c = np.zeros(max(p - 1, 1), np.int32)
+    _load().or_unrank(n, p, r, _p(c, C.c_int32))
+    return [int(x) for x in c[: p - 1]]
 
 
 def comm_ns(nbytes: int, bw: int) -> int:

@@ -114,6 +114,8 @@ def _load_lib():
     lib.ap_last_kernel_ms.argtypes = [P(C.c_float)]
     lib.ap_last_sims.restype = i32
     lib.ap_last_sims.argtypes = [P(u64)]
+    lib.ap_kernel_launches.restype = u64
+    lib.ap_kernel_launches.argtypes = []
     return lib
 
 
@@ -128,7 +130,7 @@ EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "
            "ap_last_truncated",
            "ap_decode", "ap_slice_sweep", "ap_slice_sweep_paper", "ap_slicer_alg2",
            "ap_critical_path", "ap_alg1", "ap_min_lower_bound", "ap_last_launch",
-           "ap_last_kernel_ms", "ap_last_sims")
+           "ap_last_kernel_ms", "ap_last_sims", "ap_kernel_launches")
 
 
 def _check(st: int):
@@ -412,3 +414,8 @@ def ap_last_sims() -> int:
     v = C.c_uint64()
     _check(lib.ap_last_sims(C.byref(v)))
     return int(v.value)
+
+
+def ap_kernel_launches() -> int:
+    """Kernels launched by libap.so since it was loaded (include/ap.h)."""
+    return int(lib.ap_kernel_launches())

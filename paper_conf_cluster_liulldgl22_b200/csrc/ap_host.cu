@@ -280,6 +280,8 @@ ap_status ap_last_sims(uint64_t* sims) {
   return AP_OK;
 }
 
+uint64_t ap_kernel_launches(void) { return apk::kernel_launches(); }
+
 ap_status ap_last_kernel_ms(float* ms) {
   if (!ms) return fail(AP_ERR_INVALID, "ms is NULL");
   if (!g_timer.armed) return fail(AP_ERR_INVALID, "no search launched on this thread");

@@ -14,6 +14,7 @@
 //   k_unrank, k_init    decode / key init.
 // Every kernel starts with the K4 prologue (TMA bulk copy of the tables into
 // shared memory + warp-shuffle prefix sums), see ap_device.cuh.
+#include <atomic>
 #include <climits>
 #include <cstdlib>
 #include <cstdio>
@@ -24,6 +25,12 @@
 
 namespace apk {
 using namespace apdev;
+
+// Every kernel launch of the library bumps this counter (ap_kernel_launches), so a
+// bench can state how many of its own kernels ran in a timed region.
+static std::atomic<unsigned long long> g_kernel_launches{0};
+static inline void count_launch() { g_kernel_launches.fetch_add(1, std::memory_order_relaxed); }
+unsigned long long kernel_launches() { return g_kernel_launches.load(std::memory_order_relaxed); }
 
 // ===========================================================================
 // K1 fast sweep.
@@ -453,6 +460,7 @@ __global__ void k_sweep_prep(PrepArgs a, SweepDev* out) {
 }
 
 cudaError_t launch_sweep_prep(const PrepArgs& a, SweepDev* out, cudaStream_t s) {
+  count_launch();
   k_sweep_prep<<<1, 1, 0, s>>>(a, out);
   return cudaGetLastError();
 }
@@ -2710,6 +2718,7 @@ __global__ void k_alg2(DevTables t, int p, const int32_t* cuts, int reading, int
 cudaError_t launch_alg2(const DevTables& t, int p, const int32_t* cuts, int reading, int32_t* mb,
                         cudaStream_t s) {
   const size_t smem = tables_smem_bytes(t.npad, t.n);
+  count_launch();
   k_alg2<<<1, 32, smem, s>>>(t, p, cuts, reading, mb);
   return cudaGetLastError();
 }
@@ -2757,6 +2766,7 @@ cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, 
                       (size_t)(t.n + 1) * (p + 1) * 8;
   cudaError_t e = set_smem((const void*)k_alg1, smem);
   if (e != cudaSuccess) return e;
+  count_launch();
   k_alg1<<<1, 256, smem, s>>>(t, p, arg, cuts, value);
   return cudaGetLastError();
 }
@@ -2767,6 +2777,7 @@ cudaError_t launch_minlb(const DevTables& t, int p, int m, int K, int16_t* arg, 
                       (size_t)(t.n + 1) * (p + 1) * 8;
   cudaError_t e = set_smem((const void*)k_minlb, smem);
   if (e != cudaSuccess) return e;
+  count_launch();
   k_minlb<<<1, 256, smem, s>>>(t, p, m, K, arg, cuts, value);
   return cudaGetLastError();
 }
@@ -2802,6 +2813,7 @@ static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   const int64_t wave = (int64_t)num_sms(dev) * occ;
   if (blocks > wave) blocks = wave;  // (redo pass: the listed count is <= A.count)
   if (blocks > 0) {
+    count_launch();
     k_eval<P><<<(unsigned)blocks, threads, smem, s>>>(A);
     if (launches) ++*launches;
   }
@@ -2825,6 +2837,7 @@ static cudaError_t eval_fast_P(const EvalArgs& A, cudaStream_t s, int* launches)
   const int64_t wave = (int64_t)num_sms(dev) * occ;
   if (blocks > wave) blocks = wave;
   if (blocks > 0) {
+    count_launch();
     k_eval_fast<P><<<(unsigned)blocks, threads, smem, s>>>(A);
     if (launches) ++*launches;
   }
@@ -2942,6 +2955,7 @@ static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int
     blocks = (nthreads + threads - 1) / threads;
   }
   if (A.rec && blocks > (uint64_t)sweep_max_blocks(dev)) return cudaErrorInvalidValue;
+  count_launch();
   k_sweep_exact<P, V><<<(unsigned)blocks, threads, smem, s>>>(A);
   sp->blocks = (int)blocks;
   sp->threads = threads;
@@ -2968,6 +2982,7 @@ static cudaError_t sweep_generic_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, i
   const uint64_t nthreads = (nr + A.chunk - 1) / A.chunk;
   const uint64_t blocks = (nthreads + threads - 1) / threads;
   if (A.rec && blocks > (uint64_t)sweep_max_blocks(dev)) return cudaErrorInvalidValue;
+  count_launch();
   k_sweep_generic<P><<<(unsigned)blocks, threads, smem, s>>>(A);
   sp->blocks = (int)blocks;
   sp->threads = threads;
@@ -3000,12 +3015,14 @@ static cudaError_t sweep_exact_dispatch(int p, int want_u32, const SweepArgs& A,
 
 cudaError_t launch_reduce2(const unsigned long long* rec, int nrec, long long* out,
                            cudaStream_t s) {
+  count_launch();
   k_reduce2<<<1, 256, 0, s>>>(rec, nrec, out);
   return cudaGetLastError();
 }
 
 cudaError_t launch_key2_select(const long long* local, const long long* t_star, long long* idx,
                                cudaStream_t s) {
+  count_launch();
   k_key2_select<<<1, 1, 0, s>>>(local, t_star, idx);
   return cudaGetLastError();
 }
@@ -3086,6 +3103,7 @@ static cudaError_t heur_P(const HeurArgs& A, cudaStream_t s, int dev, uint64_t n
   const uint64_t need = (nwork + threads - 1) / threads;
   if (blocks > need) blocks = need;
   if (blocks < 1) blocks = 1;
+  count_launch();
   k_heur<P, FAST><<<(unsigned)blocks, threads, smem, s>>>(A);
   return cudaGetLastError();
 }
@@ -3115,6 +3133,7 @@ static cudaError_t heur_pool_P(const HeurArgs& A, cudaStream_t s, int dev, uint6
   const uint64_t need = (nwork + hpool::NSW * hpool::NW - 1) / (hpool::NSW * hpool::NW);
   if (blocks > need) blocks = need;
   if (blocks < 1) blocks = 1;
+  count_launch();
   k_heur_pool<P><<<(unsigned)blocks, threads, smem, s>>>(A);
   return cudaGetLastError();
 }
@@ -3200,6 +3219,7 @@ static cudaError_t reach_pool_P(ReachArgs* A, cudaStream_t s, int dev, uint64_t 
   if (blocks < 1) blocks = 1;
   *lists_out = (int)blocks * RP_NS;
   if (!launch) return cudaSuccess;
+  count_launch();
   k_reach_pool<P><<<(unsigned)blocks, RP_NT, smem, s>>>(*A);
   return cudaGetLastError();
 }
@@ -3235,6 +3255,7 @@ static cudaError_t reach_P(ReachArgs* A, cudaStream_t s, int dev, uint64_t R, bo
   if (blocks < 1) blocks = 1;
   *blocks_out = (int)blocks * 32;  // one list per quad
   if (!launch) return cudaSuccess;
+  count_launch();
   k_reach<P><<<(unsigned)blocks, threads, smem, s>>>(*A);
   return cudaGetLastError();
 }
@@ -3340,6 +3361,7 @@ static cudaError_t cpath_P(CpathArgs A, cudaStream_t s) {
   const size_t smem = tables_smem_bytes(A.t.npad, A.t.n);
   cudaError_t e = set_smem((const void*)k_cpath<P>, smem);
   if (e != cudaSuccess) return e;
+  count_launch();
   k_cpath<P><<<1, 32, smem, s>>>(A);
   return cudaGetLastError();
 }
@@ -3381,6 +3403,7 @@ cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t*
 }
 
 cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s) {
+  count_launch();
   k_init_key<<<1, 1, 0, s>>>(key);
   if (counter) {
     cudaError_t e = cudaMemsetAsync(counter, 0, 3 * sizeof(unsigned int), s);  // cursors + redo count
@@ -3391,6 +3414,7 @@ cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cuda
 
 cudaError_t launch_unrank(const DevTables& t, int p, uint64_t rank, int32_t* cuts,
                           cudaStream_t s) {
+  count_launch();
   k_unrank<<<1, 32, 0, s>>>(t, p, rank, cuts);
   return cudaGetLastError();
 }

@@ -146,4 +146,7 @@ cudaError_t launch_alg2(const DevTables& t, int p, const int32_t* cuts, int read
 
 int num_sms(int device);
 
+// Kernels launched by the library since load (all threads, all devices).
+unsigned long long kernel_launches();
+
 }  // namespace apk

@@ -393,6 +393,31 @@ def test_rank_and_count(oracle_mod):
     assert oracle_mod.count(66, 8) == 696190560
 
 
+def test_unrank_and_windows(oracle_mod):
+    """The enumeration starts a rank window at the cut vector of its first rank: unrank
+    is itertools' lexicographic order (independent of the rank formula), and a search
+    split into random windows equals the single full enumeration (min over windows of
+    (T, rank, k), simulation counts summing to N*K)."""
+    for n in range(2, 11):
+        for p in range(1, n + 1):
+            for r, comb in enumerate(itertools.combinations(range(1, n), p - 1)):
+                assert oracle_mod.unrank(n, p, r) == list(comb)
+    rng = np.random.default_rng(9)
+    for seed in range(12):
+        n = 7 + seed % 6
+        f, b, a = synth.random_tables(seed, n, ["uniform", "equal", "small"][seed % 3])
+        M = oracle_mod.Model(f, b, a, synth.link_for(["uniform", "equal", "small"][seed % 3]))
+        p = 2 + seed % 4
+        m = p + seed % 3
+        N = oracle_mod.count(n, p)
+        full = M.exhaustive(p, m, 1, 3)
+        cuts = sorted({0, N, *[int(x) for x in rng.integers(0, N, 4)]})
+        parts = [M.exhaustive(p, m, 1, 3, lo, hi) for lo, hi in zip(cuts, cuts[1:]) if hi > lo]
+        best = min(parts, key=lambda d: (d["T"], d["rank"], d["k"]))
+        assert (best["T"], best["rank"], best["k"]) == (full["T"], full["rank"], full["k"])
+        assert sum(d["sims"] for d in parts) == full["sims"] == 3 * N
+
+
 def test_exhaustive_brute_force_tiny(oracle_mod):
     """or_exhaustive == min over itertools.combinations of (T, rank, k)."""
     for seed in range(40):

@@ -706,7 +706,9 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
         for (int x = 0; x < P; ++x) {
           const V Fx = sPf[c[x + 1]] - sPf[c[x]];
           const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
-          if (x == P - 2) alast = fill + (uint64_t)divk(Cin, Kh, MK) + tail;
+          if constexpr (P >= 2) {
+            if (x == P - 2) alast = fill + (uint64_t)divk(Cin, Kh, MK) + tail;
+          }
           uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
           if (x < P - 1) {
             // 1F1B bubble: B(x, 0) waits for micro-batch 0's round trip
@@ -729,7 +731,8 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
           tail += (uint64_t)wB[x];
         }
         live = xf == P;
-        if (P >= 2 && xf == P - 1) {
+        if constexpr (P >= 2) {
+        if (xf == P - 1) {
           // Only the last stage fails.  Its bound without the comm terms C_{P-2},
           // L(c) = alast + floor((Pf[c]-Pf[c_{P-2}])/K) + Pb[c]-Pb[c_{P-2}]
           //        + m*(Pf[n]-Pf[c] + Pb[n]-Pb[c]),  c = c_{P-1},
@@ -758,6 +761,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
             mono = true;
           }
         }
+        }  // P >= 2
         if (!live && (xf < P - 1 || mono)) {
           // LB_xf depends only on the prefix c_1..c_{xf+1}, so every partition with
           // that prefix is pruned too.  If the bound holds on the stage's compute alone

@@ -494,6 +494,40 @@ cudaStream_t S_(ap_stream_t s) { return reinterpret_cast<cudaStream_t>(s); }
 
 extern "C" {
 
+}  // extern "C"
+
+namespace {
+// u32 fast path of the evaluation kernel: clamping every CR rows at S
+// with (CR + p + 2) * W_row <= 2^32-1-S cannot wrap (a segment, the conversion row and
+// the p cool-down rows; from 0 the warm-up is shorter), so every candidate with T < S
+// is exact and the rest are recomputed in int64.  Used by ap_eval_batch and by every
+// internal evaluation (T_ref, decode, Slicer sweep).  AP_EVAL=int64 disables it,
+// AP_EVAL_S=<v> lowers S (tests of the fallback).
+struct EvalFast {
+  uint32_t S;
+  int CR, div1;
+};
+EvalFast eval_fast(const ap_plan* plan, int p) {
+  EvalFast ef{0, 16, 0};
+  const unsigned __int128 wrow = (unsigned __int128)(plan->sum_f + plan->sum_b) +
+                                 (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
+  const unsigned __int128 need = wrow * (unsigned __int128)(ef.CR + p + 2);
+  const unsigned __int128 lim32 = ((unsigned __int128)1 << 32) - 1;
+  ef.S = need < lim32 ? (uint32_t)(lim32 - need) : 0u;
+  const char* ev = getenv("AP_EVAL");
+  if (ev && strcmp(ev, "int64") == 0) ef.S = 0;
+  const char* es = getenv("AP_EVAL_S");
+  if (es && ef.S > 0) {
+    const unsigned long long v = strtoull(es, nullptr, 10);
+    if (v > 0 && v < ef.S) ef.S = (uint32_t)v;
+  }
+  ef.div1 = (plan->sum_f < (1ll << 28) && plan->max_comm < (1ll << 28)) ? 1 : 0;
+  return ef;
+}
+}  // namespace
+
+extern "C" {
+
 ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
                         const int32_t* k, int64_t count, int64_t* time_ns, int32_t* master,
                         ap_stream_t stream) {
@@ -507,27 +541,9 @@ ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t
   int launches = 0;
   static const int32_t kDummy = 0;
   (void)kDummy;
-  // u32 fast path: clamping every CR rows at S with
-  // (CR + p + 2) * W_row <= 2^32-1-S cannot wrap (a segment, the conversion row and the
-  // p cool-down rows; from 0 the warm-up is shorter), so every candidate with T < S is
-  // exact and the rest are recomputed in int64.  AP_EVAL=int64 disables it,
-  // AP_EVAL_S=<v> lowers S (tests of the fallback).
-  const int eCR = 16;
-  const unsigned __int128 wrow = (unsigned __int128)(plan->sum_f + plan->sum_b) +
-                                 (unsigned __int128)2 * (p - 1) * (uint64_t)plan->max_comm + 1;
-  const unsigned __int128 need = wrow * (unsigned __int128)(eCR + p + 2);
-  const unsigned __int128 lim32 = ((unsigned __int128)1 << 32) - 1;
-  uint32_t fastS = need < lim32 ? (uint32_t)(lim32 - need) : 0u;
-  const char* ev = getenv("AP_EVAL");
-  if (ev && strcmp(ev, "int64") == 0) fastS = 0;
-  const char* es = getenv("AP_EVAL_S");
-  if (es && fastS > 0) {
-    const unsigned long long v = strtoull(es, nullptr, 10);
-    if (v > 0 && v < fastS) fastS = (uint32_t)v;
-  }
-  const int div1 = (plan->sum_f < (1ll << 28) && plan->max_comm < (1ll << 28)) ? 1 : 0;
+  const EvalFast ef = eval_fast(plan, p);
   AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? cuts : nullptr, p - 1, k, 1, 0, count,
-                           time_ns, master, S_(stream), &launches, 1, 0, fastS, eCR, div1));
+                           time_ns, master, S_(stream), &launches, 1, 0, ef.S, ef.CR, ef.div1));
   return AP_OK;
 }
 
@@ -672,8 +688,11 @@ ap_status search_exhaustive_impl(const ap_plan* plan, int32_t p, int32_t m, int3
   int64_t* d_tref;
   AP_CUDA(sc.get((void**)&d_tref, 8 * (size_t)nk));
   int launches = 1;
-  AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 1, nk,
-                           d_tref, nullptr, s, &launches));
+  {
+    const EvalFast ef = eval_fast(plan, p);
+    AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_a1 : nullptr, 0, nullptr, k_lo, 1,
+                             nk, d_tref, nullptr, s, &launches, 1, 0, ef.S, ef.CR, ef.div1));
+  }
   // Everything that depends on T_ref -- S = T_ref + 1, the u32 choice, its clamp
   // schedule, the key-packing test -- is computed on the device (k_sweep_prep) and read
   // by the sweep kernels: no host synchronisation inside the search.
@@ -990,7 +1009,8 @@ ap_status ap_decode_reachable(const ap_plan* plan, int32_t p, int32_t m, uint64_
       int launches = 0;
       if (e == cudaSuccess)
         e = apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, 1,
-                             0, 1, d_T, d_master, s, &launches);
+                             0, 1, d_T, d_master, s, &launches, 1, 0, eval_fast(plan, p).S,
+                             eval_fast(plan, p).CR, eval_fast(plan, p).div1);
       int32_t hc[32] = {0};
       int64_t T = -1;
       int32_t M = -1;
@@ -1131,8 +1151,9 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
     }
     if (res == AP_OK) {
       int launches = 0;
+      const EvalFast ef = eval_fast(plan, p);
       e = apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, kk, 0, 1, d_T,
-                           d_master, s, &launches);
+                           d_master, s, &launches, 1, 0, ef.S, ef.CR, ef.div1);
       int32_t hc[32] = {0};
       int64_t T = -1;
       int32_t M = -1;
@@ -1189,7 +1210,8 @@ ap_status ap_slice_sweep(const ap_plan* plan, int32_t p, int32_t m, const int32_
     int launches = 0;
     if (e == cudaSuccess)
       e = apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? d_cuts : nullptr, 0, nullptr, 1, 1, k_max,
-                           d_T, nullptr, s, &launches);
+                           d_T, nullptr, s, &launches, 1, 0, eval_fast(plan, p).S,
+                           eval_fast(plan, p).CR, eval_fast(plan, p).div1);
     if (e == cudaSuccess)
       e = cudaMemcpyAsync(time_ns, d_T, 8 * (size_t)k_max, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);

@@ -1218,7 +1218,8 @@ AP_DEV_INLINE bool load_cuts(const int32_t* row, int p, int n, int (&c)[P + 1]) 
 template <int P>
 __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
   // the generic exact int64 evaluation (any p <= P, m, k, s); with A.redo_in set it
-  // evaluates exactly the candidates k_eval_fast listed
+  // evaluates exactly the candidates k_eval_fast listed (usually none: return at once)
+  if (A.redo_in && A.redo_in[0] == 0u) return;
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
@@ -1339,8 +1340,8 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
 // Algorithm 1, one CTA.  time[0][0] = 0, others +inf;
 // time[i][j] = min_k max(time[k][j-1], P[i]-P[k]) over k ascending, strict '<'
 // (smallest k wins ties); the arg table drives line 15's reconstruction.
-__global__ void __launch_bounds__(256) k_alg1(DevTables t, int p, int16_t* arg, int32_t* cuts,
-                                              int64_t* value) {
+__global__ void __launch_bounds__(1024) k_alg1(DevTables t, int p, int16_t* arg, int32_t* cuts,
+                                               int64_t* value) {
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(t.tab, t.n, t.npad, smem, &used);
@@ -1352,14 +1353,16 @@ __global__ void __launch_bounds__(256) k_alg1(DevTables t, int p, int16_t* arg, 
     arg[e] = -1;
   }
   __syncthreads();
+  // time[i][j] reads only column j-1, so the columns go one after another and every i of
+  // a column in parallel (a warp per i, lanes over k): p dependent steps instead of n.
+  // Same values and the same argmin as the paper's i-outer loop (smallest k on ties).
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31, nw = blockDim.x >> 5;
-  for (int i = 1; i <= n; ++i) {
-    const int64_t Pi = T.Pf[i] + T.Pb[i];
-    const int jmax = min(p, i);
-    for (int j = 1 + warp; j <= jmax; j += nw) {
+  for (int j = 1; j <= p; ++j) {
+    for (int i = j + warp; i <= n; i += nw) {
+      const int64_t Pi = T.Pf[i] + T.Pb[i];
       int64_t bv = INT64_MAX;
       int bk = INT32_MAX;
-      for (int kk = lane; kk <= i - 1; kk += 32) {
+      for (int kk = j - 1 + lane; kk <= i - 1; kk += 32) {
         const int64_t prev = tt[kk * P1 + (j - 1)];
         const int64_t seg = Pi - (T.Pf[kk] + T.Pb[kk]);
         const int64_t v = prev > seg ? prev : seg;
@@ -1514,6 +1517,8 @@ AP_DEV_INLINE void alg1_prefix(const int16_t* s_arg, int P1, int c, int j, int* 
 // sim_exact (runtime p <= P), over [r_lo, r_hi) or over the ids listed in A.redo.
 template <int P, bool FAST>
 __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
+  // the exact redo pass over the restarts the u32 pass abandoned (usually none)
+  if (!FAST && A.redo && A.redo[0] == 0u) return;
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
@@ -2728,23 +2733,39 @@ cudaError_t launch_alg2(const DevTables& t, int p, const int32_t* cuts, int read
 }
 
 __global__ void k_unrank(DevTables t, int p, uint64_t rank, int32_t* cuts) {
-  if (threadIdx.x != 0 || blockIdx.x != 0) return;
-  const int n = t.n;
+  // one warp: c_x = the least v > c_{x-1} with rank < sum_{u=c_{x-1}+1}^{v} C(n-1-u, p-1-x)
+  // (reading O7), 32 candidate v per step with a warp prefix sum
+  if (blockIdx.x != 0 || threadIdx.x >= 32) return;
+  const int n = t.n, lane = threadIdx.x;
   uint64_t rr = rank;
   int prev = 0;
   for (int x = 1; x <= p - 1; ++x) {
-    int v = prev + 1;
+    int base = prev + 1;
     for (;;) {
-      const uint64_t cnt = binom_at(t.binom, n - 1 - v, p - 1 - x);
-      if (rr >= cnt) {
-        rr -= cnt;
-        ++v;
-      } else {
+      const int v = base + lane;
+      uint64_t c = (v <= n - 1) ? binom_at(t.binom, n - 1 - v, p - 1 - x) : 0ull;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {  // inclusive prefix sum over the 32 candidates
+        const uint64_t u = __shfl_up_sync(0xffffffffu, c, o);
+        if (lane >= o) c += u;
+      }
+      // the first lane whose running sum exceeds rr holds c_x
+      const unsigned int hit = __ballot_sync(0xffffffffu, c > rr);
+      if (hit) {
+        const int l = __ffs(hit) - 1;
+        const uint64_t below = __shfl_sync(0xffffffffu, c, l > 0 ? l - 1 : 0);
+        if (l > 0) rr -= below;
+        prev = base + l;
+        break;
+      }
+      rr -= __shfl_sync(0xffffffffu, c, 31);
+      base += 32;
+      if (base > n) {  // rank beyond C(n-1, p-1): the caller validated it, cannot happen
+        prev = n;
         break;
       }
     }
-    cuts[x - 1] = v;
-    prev = v;
+    if (lane == 0) cuts[x - 1] = prev;
   }
 }
 
@@ -2771,7 +2792,7 @@ cudaError_t launch_alg1(const DevTables& t, int p, int16_t* arg, int32_t* cuts, 
   cudaError_t e = set_smem((const void*)k_alg1, smem);
   if (e != cudaSuccess) return e;
   count_launch();
-  k_alg1<<<1, 256, smem, s>>>(t, p, arg, cuts, value);
+  k_alg1<<<1, 1024, smem, s>>>(t, p, arg, cuts, value);
   return cudaGetLastError();
 }
 

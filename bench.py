@@ -565,6 +565,32 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
     out["C3"] = {"workload": wl.name, "sims_per_s": N / (float(t[0]) / 1e3),
                  "time_to_optimal_plan_ms": float(t[0]), "T_ns": r3["time_ns"], "cuts": r3["cuts"]}
+    # the pruned exact search (same key) captured once in a CUDA graph and replayed: the
+    # search is stream-ordered end to end (no host synchronisation inside it)
+    try:
+        gk = torch.empty(1, dtype=torch.int64, device=dev)
+        side = torch.cuda.Stream()
+        side.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(side):
+            ap.ap_search_exhaustive_mode(plan, wl.p, wl.m, 1, 1, lo, hi, ap.AP_SEARCH_PRUNED, gk)
+        torch.cuda.current_stream().wait_stream(side)
+        torch.cuda.synchronize()
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            ap.ap_search_exhaustive_mode(plan, wl.p, wl.m, 1, 1, lo, hi, ap.AP_SEARCH_PRUNED, gk)
+        graph.replay()
+        torch.cuda.synchronize()
+        times = []
+        for _ in range(10):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(); graph.replay(); e1.record(); torch.cuda.synchronize()
+            times.append(e0.elapsed_time(e1))
+        if world > 1:
+            dist.all_reduce(gk, op=dist.ReduceOp.MIN)
+        out["C3"]["pruned_search_graph_replay_ms"] = statistics.median(times)
+        out["C3"]["pruned_graph_key_equals_full"] = int(gk.item()) == int(key.item())
+    except Exception as e:  # a capture failure is reported, not hidden
+        out["C3"]["pruned_search_graph_error"] = repr(e)
     # C5
     wl = synth.config(5)
     f, b, a = wl.arrays()

@@ -1215,7 +1215,9 @@ AP_DEV_INLINE bool load_cuts(const int32_t* row, int p, int n, int (&c)[P + 1]) 
   return ok;
 }
 
-template <int P>
+// SLICED = true: the paper's Slicer form (s != 1 leading micro-batches sliced, T only),
+// in a kernel of its own so its per-piece arrays do not weigh on the common one.
+template <int P, bool SLICED>
 __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
   // the generic exact int64 evaluation (any p <= P, m, k, s); with A.redo_in set it
   // evaluates exactly the candidates k_eval_fast listed (usually none: return at once)
@@ -1242,7 +1244,7 @@ __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
     }
     int64_t F[P], B[P], C[P];
     stage_costs<P>(T, p, c, F, B, C);
-    if (sl != 1) {  // paper Slicer form: T only
+    if constexpr (SLICED) {  // paper Slicer form: T only
       A.time_ns[i] = sim_sliced<P>(p, m, sl, k, F, B, C);
       if (A.master) A.master[i] = -1;
       continue;
@@ -2826,12 +2828,14 @@ static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
       smem = base + per * threads;
     }
   }
-  cudaError_t e = set_smem((const void*)k_eval<P>, smem);
+  const bool sliced = A.s_iota || A.s_const != 1;
+  const void* fn = sliced ? (const void*)k_eval<P, true> : (const void*)k_eval<P, false>;
+  cudaError_t e = set_smem(fn, smem);
   if (e != cudaSuccess) return e;
   // persistent grid: at most one wave (the kernel strides over the candidates)
   int occ = 0, dev = 0;
   cudaGetDevice(&dev);
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval<P>, threads, smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem);
   if (e != cudaSuccess) return e;
   occ = occ < 1 ? 1 : occ;
   int64_t blocks = (A.count + threads - 1) / threads;
@@ -2839,7 +2843,10 @@ static cudaError_t eval_P(const EvalArgs& A0, cudaStream_t s, int* launches) {
   if (blocks > wave) blocks = wave;  // (redo pass: the listed count is <= A.count)
   if (blocks > 0) {
     count_launch();
-    k_eval<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+    if (sliced)
+      k_eval<P, true><<<(unsigned)blocks, threads, smem, s>>>(A);
+    else
+      k_eval<P, false><<<(unsigned)blocks, threads, smem, s>>>(A);
     if (launches) ++*launches;
   }
   return cudaGetLastError();

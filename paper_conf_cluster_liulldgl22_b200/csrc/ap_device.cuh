@@ -25,6 +25,7 @@ namespace apdev {
 
 constexpr int kMaxP = 32;
 constexpr int kMaxK = 16;
+constexpr int kMaxN = 512;  // AP_MAX_N
 
 AP_DEV_INLINE uint32_t smem_addr(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));

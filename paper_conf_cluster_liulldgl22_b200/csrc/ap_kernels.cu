@@ -214,7 +214,19 @@ AP_DEV_INLINE void pieces(int k, const V (&wF)[P], const int (&c)[P + 1], const 
 // a clamp every `every` steady rows, and `fin` = clamp once more at the end of the
 // steady rows.  Ignored for 64-bit V.
 struct ClampSched {
-  int first, every, fin;
+  int first_, every_, fin_;
+  AP_DEV_INLINE int first() const { return first_; }
+  AP_DEV_INLINE int every() const { return every_; }
+  AP_DEV_INLINE int fin() const { return fin_; }
+};
+// The exhaustive sweep's schedule lives in the device record k_sweep_prep wrote; it is
+// read where it is used (volatile: one L1 load per use) instead of being held in three
+// registers for the whole kernel, which had pushed k_sweep_exact<8,u32> into spills.
+struct ClampDev {
+  const int* p;  // &SweepDev::clamp_first (then clamp_rows, clamp_final)
+  AP_DEV_INLINE int first() const { return *reinterpret_cast<const volatile int*>(p); }
+  AP_DEV_INLINE int every() const { return *reinterpret_cast<const volatile int*>(p + 1); }
+  AP_DEV_INLINE int fin() const { return *reinterpret_cast<const volatile int*>(p + 2); }
 };
 
 // Everything after the pieces, for p == P, m >= P: warm-up rows, the first 1F1B row,
@@ -228,9 +240,9 @@ struct ClampSched {
 //        G[x] = B'(x, m-2) for x <= P-2 (longest path from the end of F(x,0) via
 //               F(x,1)),   G[P-1] = F'(P-1, m-1) (via B(P-1,0)),
 //      so that T(k) = max_x (FF_x(k) + G[x]) for every k.
-template <int P, typename V, bool REV>
+template <int P, typename V, bool REV, typename CS>
 AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V S,
-                           ClampSched cs, uint32_t one, V (&G)[P]) {
+                           CS cs, uint32_t one, V (&G)[P]) {
   using O = XOps<V>;
   V L[P];
   // warm-up rows r = 1..P-2: stage x <= r-1 does F(x, r-x); L == FF here
@@ -252,8 +264,8 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
     constexpr int U = (P <= 8) ? 8 : 4;
     const V wBF0 = wB[0] + wF[0];
     int rem = m - P;
-    if (sizeof(V) == 4 && cs.first == 0) clamp_ff<P, V>(FF, S);
-    int seg = (sizeof(V) == 4 && cs.first > 0) ? cs.first : cs.every;
+    if (sizeof(V) == 4 && cs.first() == 0) clamp_ff<P, V>(FF, S);
+    int seg = (sizeof(V) == 4 && cs.first() > 0) ? cs.first() : cs.every();
     if (sizeof(V) != 4) seg = rem;
     if constexpr (P >= 3 && AP_NFORM) {
       if (rem > 0) {
@@ -293,12 +305,12 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
           }
           if (rem <= 0) break;
           clamp_n<P, V>(N, S);
-          blk = rem < cs.every ? rem : cs.every;
+          blk = rem < cs.every() ? rem : cs.every();
           rem -= blk;
         }
         // back to finishes (u32: FF = N + c sits up to one row's growth above N, which
         // the host's clamp_final test allows for: last segment + 1 + p rows)
-        if (cs.fin) clamp_n<P, V>(N, S);
+        if (cs.fin()) clamp_n<P, V>(N, S);
 #pragma unroll
         for (int x = 0; x <= P - 2; ++x) FF[x + 1] = fma_add(N[x], c[x + 1], one);
         FF[0] = fma_add(N[0], fma_add(c[0], sw[0], one), one);
@@ -313,10 +325,10 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
         for (int u = 0; u < U; ++u) mstep<P, V>(FF, wF, wB, wBF0, one);
       }
       for (; blk > 0; --blk) mstep<P, V>(FF, wF, wB, wBF0, one);
-      if (rem > 0 || cs.fin) clamp_ff<P, V>(FF, S);
-      seg = cs.every;
+      if (rem > 0 || cs.fin()) clamp_ff<P, V>(FF, S);
+      seg = cs.every();
     }
-    if (m == P && cs.fin && cs.first != 0) clamp_ff<P, V>(FF, S);
+    if (m == P && cs.fin() && cs.first() != 0) clamp_ff<P, V>(FF, S);
   }
   // cool-down, fused the same way: step t = 0..P-1 is the backward pass of row
   // r = m-1+t plus the forward pass of row r+1, which only stages x >= t+1 still
@@ -359,10 +371,10 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
 }
 
 // Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
-template <int P, typename V>
+template <int P, typename V, typename CS>
 AP_DEV_INLINE V sim_fast(int m, int k, const V (&wF)[P], const V (&wB)[P], const int (&c)[P + 1],
                          const V* sPf, const V* sC, uint32_t Mk, bool div1, V S,
-                         ClampSched cs, uint32_t one) {
+                         CS cs, uint32_t one) {
   V FF[P], G[P];
   pieces<P, V>(k, wF, c, sPf, sC, Mk, div1, one, FF);
   return sweep_tail<P, V, false>(m, FF, wF, wB, S, cs, one, G);
@@ -580,13 +592,16 @@ __global__ void k_key2_select(const long long* local, const long long* t_star, l
                                                                     : 0x7fffffffffffffffll;
 }
 
-template <int P, typename V>
+template <int P, typename V, bool FACT>
 __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1, V S,
-                                            ClampSched cs, const V* sPf, const V* sPb,
+                                            ClampDev cs, const V* sPf, const V* sPb,
                                             const V* sC, const uint32_t* s_mk, V& bestT,
                                             uint64_t& bestIdx);
 
-template <int P, typename V>
+// FACT = false: the FULL mode (every (partition, k) pair swept); FACT = true: the
+// k-factored and pruned modes.  Separate instances, so the full sweep's register
+// allocation does not carry the pruned mode's bound and re-rank code.
+template <int P, typename V, bool FACT>
 #ifndef AP_SWEEP_MINB
 #define AP_SWEEP_MINB (P <= 8 ? 3 : 2)
 #endif
@@ -596,15 +611,18 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
   const int d_u32 = A.dp->u32, d_skip = A.dp->skip;
   if (d_skip || d_u32 != A.is_u32) return;
   const uint64_t dS = A.dp->S;
-  const ClampSched dcs{A.dp->clamp_first, A.dp->clamp_rows, A.dp->clamp_final};
+  const ClampDev dcs{&A.dp->clamp_first};
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
   const int n = A.t.n;
-  // V-typed copies of the prefix sums / comm (u32 path: exact by the host's bound)
-  V* sPf = reinterpret_cast<V*>(smem + used);
-  V* sPb = sPf + (n + 1);
-  V* sC = sPb + (n + 1);
+  // V-typed copies of the prefix sums / comm (u32 path: exact by the host's bound), in
+  // a static shared array: fixed shared addresses, no pointer registers (80 registers
+  // are all the sweep has at 3 CTAs per SM)
+  __shared__ V s_tabV[3 * (kMaxN + 1)];
+  V* sPf = s_tabV;
+  V* sPb = s_tabV + (kMaxN + 1);
+  V* sC = s_tabV + 2 * (kMaxN + 1);
   __shared__ uint32_t s_mk[kMaxK + 1];  // floor(2^32 / k) (k = 1: 2^32 - 1), see divk
   for (int i = threadIdx.x; i <= n; i += blockDim.x) {
     sPf[i] = (V)T.Pf[i];
@@ -633,21 +651,21 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
       if (u * 32ull >= (span + A.chunk - 1) / A.chunk) break;
       const uint64_t r0 = A.rank_lo + (u * 32ull + (uint64_t)lane) * A.chunk;
       if (r0 < A.rank_hi)
-        sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), S, dcs, sPf, sPb, sC, s_mk, bestT, bestIdx);
+        sweep_range<P, V, FACT>(A, r0, min(r0 + A.chunk, A.rank_hi), S, dcs, sPf, sPb, sC, s_mk, bestT, bestIdx);
     }
   } else {
     const uint64_t tid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const uint64_t r0 = A.rank_lo + tid * A.chunk;
     if (r0 < A.rank_hi)
-      sweep_range<P, V>(A, r0, min(r0 + A.chunk, A.rank_hi), S, dcs, sPf, sPb, sC, s_mk, bestT, bestIdx);
+      sweep_range<P, V, FACT>(A, r0, min(r0 + A.chunk, A.rank_hi), S, dcs, sPf, sPb, sC, s_mk, bestT, bestIdx);
   }
   sweep_result(A, bestT < S, (uint64_t)bestT, bestIdx);
 }
 
 // Ranks [r0, r1) x k of one thread: unrank r0, then lex successors (a2-a7).
-template <int P, typename V>
+template <int P, typename V, bool FACT>
 __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1, V S,
-                                            ClampSched cs, const V* sPf, const V* sPb,
+                                            ClampDev cs, const V* sPf, const V* sPb,
                                             const V* sC, const uint32_t* s_mk, V& bestT,
                                             uint64_t& bestIdx) {
   const int n = A.t.n;
@@ -691,7 +709,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
       }
       const uint64_t base = r * K;
       bool live = true;
-      if (A.mode == 2) {
+      if (FACT && A.mode == 2) {
         // SURVEY O11 lower bound for every k <= k_hi (pinned by the oracle's P6):
         // LB_x = fill_x + m*(F_x+B_x+C_in+C_out) + sum_{i<x}(B_i+C_i), fill_x =
         // sum_{i<x} floor(F_i/K) + sum_{i<x-1} floor(C_i/K).  A partition with LB >= S
@@ -706,9 +724,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
         for (int x = 0; x < P; ++x) {
           const V Fx = sPf[c[x + 1]] - sPf[c[x]];
           const V Cin = (x > 0) ? sC[c[x] - 1] : V(0);
-          if constexpr (P >= 2) {
-            if (x == P - 2) alast = fill + (uint64_t)divk(Cin, Kh, MK) + tail;
-          }
+          if (x == P - 2) alast = fill + (uint64_t)divk(Cin, Kh, MK) + tail;
           uint64_t v = fill + (uint64_t)m * ((uint64_t)wF[x] + (uint64_t)wB[x]) + tail;
           if (x < P - 1) {
             // 1F1B bubble: B(x, 0) waits for micro-batch 0's round trip
@@ -731,15 +747,16 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
           tail += (uint64_t)wB[x];
         }
         live = xf == P;
-        if constexpr (P >= 2) {
-        if (xf == P - 1) {
+        // (P >= 2: the P = 1 instance never runs this block; its indices are clamped so
+        // it does not even name c[-1])
+        if (P >= 2 && xf == P - 1) {
           // Only the last stage fails.  Its bound without the comm terms C_{P-2},
           // L(c) = alast + floor((Pf[c]-Pf[c_{P-2}])/K) + Pb[c]-Pb[c_{P-2}]
           //        + m*(Pf[n]-Pf[c] + Pb[n]-Pb[c]),  c = c_{P-1},
           // is <= LB_{P-1} and non-increasing in c (one more sub-layer (f,b) adds at most
           // f + b and removes m*(f+b)), so the failing c form a prefix of [c_{P-2}+1, n-1]:
           // step c_{P-1} past it in shared memory instead of one rank at a time.
-          const int cl = c[P - 2];
+          const int cl = c[P >= 2 ? P - 2 : 0];
           auto L = [&](int cc) -> uint64_t {
             return alast + (uint64_t)divk(V(sPf[cc] - sPf[cl]), Kh, MK) + (uint64_t)(sPb[cc] - sPb[cl]) +
                    (uint64_t)m * ((uint64_t)(sPf[n] - sPf[cc]) + (uint64_t)(sPb[n] - sPb[cc]));
@@ -761,7 +778,6 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
             mono = true;
           }
         }
-        }  // P >= 2
         if (!live && (xf < P - 1 || mono)) {
           // LB_xf depends only on the prefix c_1..c_{xf+1}, so every partition with
           // that prefix is pruned too.  If the bound holds on the stage's compute alone
@@ -790,7 +806,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
           continue;
         }
       }
-      if (live && A.mode == 0) {
+      if (!FACT) {
         for (int k = k_lo; k <= k_hi; ++k) {
           const uint32_t Mk = s_mk[k];
           const V Tc = sim_fast<P, V>(m, k, wF, wB, c, sPf, sC, Mk, A.div1 != 0, S, cs, A.one);
@@ -799,7 +815,7 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
             bestIdx = base + (uint64_t)(k - k_lo);
           }
         }
-      } else if (live) {
+      } else if (live) {  // FACT
         // k-factored: one reversed sweep gives G, then T(k) = max_x FF_x(k) + G_x
         V G[P];
         if constexpr (P >= 2) {
@@ -2947,13 +2963,14 @@ int sweep_max_blocks(int dev);
 
 template <int P, typename V>
 static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int dev) {
-  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n) + (size_t)(3 * (A.t.n + 1) + 4) * sizeof(V);
-  const void* fn = (const void*)k_sweep_exact<P, V>;
+  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n);
+  const bool fact = A.mode != 0;
+  const void* fn = fact ? (const void*)k_sweep_exact<P, V, true> : (const void*)k_sweep_exact<P, V, false>;
   cudaError_t e = set_smem(fn, smem);
   if (e != cudaSuccess) return e;
   const int threads = 256;
   int occ = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_sweep_exact<P, V>, threads, smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem);
   if (e != cudaSuccess) return e;
   occ = occ < 1 ? 1 : occ;
   const uint64_t nr = A.rank_hi - A.rank_lo;
@@ -2988,7 +3005,10 @@ static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int
   }
   if (A.rec && blocks > (uint64_t)sweep_max_blocks(dev)) return cudaErrorInvalidValue;
   count_launch();
-  k_sweep_exact<P, V><<<(unsigned)blocks, threads, smem, s>>>(A);
+  if (fact)
+    k_sweep_exact<P, V, true><<<(unsigned)blocks, threads, smem, s>>>(A);
+  else
+    k_sweep_exact<P, V, false><<<(unsigned)blocks, threads, smem, s>>>(A);
   sp->blocks = (int)blocks;
   sp->threads = threads;
   sp->chunk = A.chunk;

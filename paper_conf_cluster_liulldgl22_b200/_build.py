@@ -14,11 +14,16 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
          "-cudart", "shared"]
-# AP_FAST_BUILD=1 compiles the device code in parallel (--split-compile) for quick
-# iteration.  Not the default: split compilation changes ptxas's register allocation of
-# k_sweep_exact<8, u32> (96 B of spills instead of 16 B), so release builds are whole.
-if os.environ.get("AP_FAST_BUILD") == "1":
-    FLAGS += ["--split-compile", str(max(1, min(16, os.cpu_count() or 1)))]
+# The device code is compiled as 8 NVVM partitions (--split-compile 8, a FIXED count so
+# the code does not depend on the build host's core count).  Measured on B200
+# (profiles/r02_split_compile.md): k_sweep_exact<8,u32,FULL> runs C4 in 205.7 ms this
+# way against 210.5 ms as one partition -- the whole-module build puts 46 more IMADs in
+# the per-k loop.  The partitioned build has 60 STL / 84 LDL in that kernel, all
+# outside the per-k loop (once per partition, i.e. per 8 simulations, L1-resident);
+# its row loops and per-k loop have none.  AP_SPLIT_COMPILE=0 builds one partition.
+_SPLIT = os.environ.get("AP_SPLIT_COMPILE", "8")
+if _SPLIT != "0":
+    FLAGS += ["--split-compile", _SPLIT]
 
 
 def _stale() -> bool:

@@ -219,15 +219,6 @@ struct ClampSched {
   AP_DEV_INLINE int every() const { return every_; }
   AP_DEV_INLINE int fin() const { return fin_; }
 };
-// The exhaustive sweep's schedule lives in the device record k_sweep_prep wrote; it is
-// read where it is used (volatile: one L1 load per use) instead of being held in three
-// registers for the whole kernel, which had pushed k_sweep_exact<8,u32> into spills.
-struct ClampDev {
-  const int* p;  // &SweepDev::clamp_first (then clamp_rows, clamp_final)
-  AP_DEV_INLINE int first() const { return *reinterpret_cast<const volatile int*>(p); }
-  AP_DEV_INLINE int every() const { return *reinterpret_cast<const volatile int*>(p + 1); }
-  AP_DEV_INLINE int fin() const { return *reinterpret_cast<const volatile int*>(p + 2); }
-};
 
 // Everything after the pieces, for p == P, m >= P: warm-up rows, the first 1F1B row,
 // the fused steady steps and the fused cool-down.
@@ -594,7 +585,7 @@ __global__ void k_key2_select(const long long* local, const long long* t_star, l
 
 template <int P, typename V, bool FACT>
 __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1, V S,
-                                            ClampDev cs, const V* sPf, const V* sPb,
+                                            ClampSched cs, const V* sPf, const V* sPb,
                                             const V* sC, const uint32_t* s_mk, V& bestT,
                                             uint64_t& bestIdx);
 
@@ -611,18 +602,17 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
   const int d_u32 = A.dp->u32, d_skip = A.dp->skip;
   if (d_skip || d_u32 != A.is_u32) return;
   const uint64_t dS = A.dp->S;
-  const ClampDev dcs{&A.dp->clamp_first};
+  // (held in registers: re-reading it through memory at each use cost 26% on C4,
+  // profiles/r02_split_compile.md)
+  const ClampSched dcs{A.dp->clamp_first, A.dp->clamp_rows, A.dp->clamp_final};
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
   const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
   const int n = A.t.n;
-  // V-typed copies of the prefix sums / comm (u32 path: exact by the host's bound), in
-  // a static shared array: fixed shared addresses, no pointer registers (80 registers
-  // are all the sweep has at 3 CTAs per SM)
-  __shared__ V s_tabV[3 * (kMaxN + 1)];
-  V* sPf = s_tabV;
-  V* sPb = s_tabV + (kMaxN + 1);
-  V* sC = s_tabV + 2 * (kMaxN + 1);
+  // V-typed copies of the prefix sums / comm (u32 path: exact by the host's bound)
+  V* sPf = reinterpret_cast<V*>(smem + used);
+  V* sPb = sPf + (n + 1);
+  V* sC = sPb + (n + 1);
   __shared__ uint32_t s_mk[kMaxK + 1];  // floor(2^32 / k) (k = 1: 2^32 - 1), see divk
   for (int i = threadIdx.x; i <= n; i += blockDim.x) {
     sPf[i] = (V)T.Pf[i];
@@ -665,7 +655,7 @@ __global__ void __launch_bounds__(256, AP_SWEEP_MINB) k_sweep_exact(SweepArgs A)
 // Ranks [r0, r1) x k of one thread: unrank r0, then lex successors (a2-a7).
 template <int P, typename V, bool FACT>
 __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uint64_t r1, V S,
-                                            ClampDev cs, const V* sPf, const V* sPb,
+                                            ClampSched cs, const V* sPf, const V* sPb,
                                             const V* sC, const uint32_t* s_mk, V& bestT,
                                             uint64_t& bestIdx) {
   const int n = A.t.n;
@@ -2963,7 +2953,7 @@ int sweep_max_blocks(int dev);
 
 template <int P, typename V>
 static cudaError_t sweep_exact_P(SweepArgs A, cudaStream_t s, SweepPlan* sp, int dev) {
-  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n);
+  const size_t smem = tables_smem_bytes(A.t.npad, A.t.n) + (size_t)(3 * (A.t.n + 1) + 4) * sizeof(V);
   const bool fact = A.mode != 0;
   const void* fn = fact ? (const void*)k_sweep_exact<P, V, true> : (const void*)k_sweep_exact<P, V, false>;
   cudaError_t e = set_smem(fn, smem);

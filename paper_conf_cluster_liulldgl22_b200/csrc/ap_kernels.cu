@@ -1305,7 +1305,12 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
                                   : (uint32_t)((1ull << 32) / threadIdx.x);
   off += eval_fast_smem(n);
   __syncthreads();
-  const Bits16 br{reinterpret_cast<uint16_t*>(smem + off) + threadIdx.x, (int)blockDim.x};
+  off = (off + 15) & ~size_t(15);
+  uint32_t* s_cw = reinterpret_cast<uint32_t*>(smem + off);
+  const MasterBits br{s_cw + threadIdx.x,
+                      reinterpret_cast<uint16_t*>(s_cw + (size_t)master_col_words(m, P) * blockDim.x) +
+                          threadIdx.x,
+                      (int)blockDim.x};
   const uint32_t S = A.fastS, one = A.one;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < A.count;
        i += (int64_t)gridDim.x * blockDim.x) {
@@ -1333,10 +1338,10 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
         done = true;
       }
     } else if (k == 1 && m <= 127) {
-      const uint32_t t32 = sim_bits16<P>(m, wF, wB, S, A.CR, br, one);
+      const uint32_t t32 = sim_master<P>(m, wF, wB, S, A.CR, br, one);
       if (t32 < S) {
         A.time_ns[i] = (int64_t)t32;
-        A.master[i] = backtrack_rows<P, 8>(m, br);
+        A.master[i] = backtrack_master<P, 8>(m, br);
         done = true;
       }
     }
@@ -1777,7 +1782,7 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
 // warp owns NSW restart slots: lane l < NSW advances slot l's walk (reading O9, in
 // exactly k_heur's order) and queues its simulation jobs -- the start, or the up to
 // four children a, a', b, b' of a step -- in the warp's ring; then each of the 32
-// lanes simulates one queued job (sim_bits16 + backtrack_rows, ap_master.cuh), all in
+// lanes simulates one queued job (sim_master + backtrack_master, ap_master.cuh), all in
 // step.  A slot whose jobs are all done advances at the next pass; free slots refill
 // from the global restart cursor.  Only __syncwarp: the warps of a CTA never wait for
 // each other.
@@ -1834,7 +1839,7 @@ __global__ void __launch_bounds__(hpool::NT, 4) k_heur_pool(HeurArgs A) {
   uint32_t* s32Pf = reinterpret_cast<uint32_t*>(s_a1 + 32);
   uint32_t* s32Pb = s32Pf + (n + 1);
   uint32_t* s32C = s32Pb + (n + 1);
-  uint16_t* s_bits = reinterpret_cast<uint16_t*>(s32C + ((n + 3) & ~3));
+  uint32_t* s_cw = s32C + ((n + 3) & ~3);  // the master bits (MasterBits)
   // per-warp slot state: cut vectors [slot][0 cur | 1 best][P+1]; a job is a slot and a
   // code (0-3: child a, a', b, b' of cur, 4: cur itself), and the lane that simulates it
   // rebuilds the child in its own scratch vector (s_scr) from cur
@@ -1856,7 +1861,8 @@ __global__ void __launch_bounds__(hpool::NT, 4) k_heur_pool(HeurArgs A) {
     if (e < n) s32C[e] = (uint32_t)T.comm[e];
   }
   __syncthreads();
-  const Bits16 br{s_bits + tid, NT};
+  const MasterBits br{s_cw + tid, reinterpret_cast<uint16_t*>(s_cw + (size_t)master_col_words(m, P) * NT) + tid,
+                      NT};
   int16_t* scr = s_scr[w][lane];
   const int smax = n * p;
   const uint32_t one = A.CR > 0 ? 1u : 0u;  // = 1, not a compile-time constant
@@ -2023,13 +2029,13 @@ __global__ void __launch_bounds__(hpool::NT, 4) k_heur_pool(HeurArgs A) {
         wF[x] = (s32Pf[c[x + 1]] - s32Pf[c[x]]) + ((x > 0) ? s32C[c[x] - 1] : 0u);
         wB[x] = (s32Pb[c[x + 1]] - s32Pb[c[x]]) + ((x < P - 1) ? s32C[c[x + 1] - 1] : 0u);
       }
-      const uint32_t t32 = sim_bits16<P>(m, wF, wB, A.S, A.CR, br, one);
+      const uint32_t t32 = sim_master<P>(m, wF, wB, A.S, A.CR, br, one);
       const int ri = code & 3;  // the start's result goes to index 0
       if (t32 >= A.S) {
         s_aband[w][sl] = 1;
       } else {
         s_chT[w][sl][ri] = t32;
-        s_chM[w][sl][ri] = (int8_t)backtrack_rows<P, 8>(m, br);
+        s_chM[w][sl][ri] = (int8_t)backtrack_master<P, 8>(m, br);
       }
       atomicSub(&s_pend[w][sl], 1);
     }
@@ -2862,8 +2868,8 @@ template <int P>
 static cudaError_t eval_fast_P(const EvalArgs& A, cudaStream_t s, int* launches) {
   const int threads = 128;
   const size_t smem = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
-                      eval_fast_smem(A.t.n) +
-                      (A.master ? (size_t)bits16_words(A.m, P) * 2 * threads : 0);
+                      ((eval_fast_smem(A.t.n) + 15) & ~size_t(15)) +
+                      (A.master ? master_bits_bytes(A.m, P, threads) : 0);
   cudaError_t e = set_smem((const void*)k_eval_fast<P>, smem);
   if (e != cudaSuccess) return e;
   int occ = 0, dev = 0;
@@ -3157,7 +3163,7 @@ static cudaError_t heur_pool_P(const HeurArgs& A, cudaStream_t s, int dev, uint6
   const size_t base = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
                       ((narg + 7) & ~size_t(7)) * 2 + 32 * 4 +
                       (size_t)(2 * (A.t.n + 1) + ((A.t.n + 3) & ~3)) * 4;
-  const size_t smem = base + (size_t)bits16_words(A.m, P) * 2 * threads;
+  const size_t smem = base + master_bits_bytes(A.m, P, threads);
   // the static slot state plus the dynamic part can pass 48 KB while the dynamic part
   // alone does not, so the attribute is always set
   cudaError_t e = cudaFuncSetAttribute((const void*)k_heur_pool<P>,

@@ -1,35 +1,45 @@
 // ap_master.cuh -- the u32 fast path WITH the master stage (k = 1, p == P <= 16,
-// P <= m <= 127): decision words written during the offset-form sweep, and a
-// run-length backtrack of the critical path (readings Q10, Q11).
+// P <= m <= 127): decision bits written during the offset-form sweep, and a walk of
+// the critical path back from the sink (readings Q10, Q11).
 //
 // Shares nothing with oracle/.  Used by k_eval_fast (ap_eval_batch with master) and
-// the heuristic's warp pool (k_heur_wpool).  DESIGN.md §5.5.
+// the heuristic's warp pool (k_heur_pool).  DESIGN.md §5.5.
 //
-// Decision words, one simulation (rows r = 0 .. m+P-2 of the row formulation,
-// ap_device.cuh: F(x, j) sits in row j + x, B(x, y) in row y + P - 1):
-//   fw[r]  (uint16) F bits: bit x (1 <= x <= P-1) = "F(x) of row r takes its cross
-//          predecessor F(x-1)" (cross > intra strictly: the intra-stage predecessor
-//          outranks on a tie, Q10).  Bit 0 and bits >= P are 0.
-//   bw[t]  (uint16) B bits of the cool-down row m-1+t, t = 0..P-1, for the stages x < t
-//          only: bit x = "B(x) takes its cross predecessor B(x+1)" (cross >= intra:
-//          the cross one, stage x+1, outranks on a tie).
+// Decision bits of one simulation (row formulation of ap_device.cuh: F(x, j) sits in
+// row j + x, B(x, y) in row y + P - 1):
+//   F bit (x, r), 1 <= x <= P-1: "F(x) of row r takes its cross predecessor F(x-1)"
+//          (cross > intra strictly: the intra-stage predecessor outranks on a tie, Q10).
+//   B bit (x, t) of the cool-down row m-1+t, t = 0..P-1, stages x < t only: "B(x)
+//          takes its cross predecessor B(x+1)" (cross >= intra: stage x+1 outranks on
+//          a tie).
 // Every other B bit is NOT stored: wherever stage x still runs a forward in row r+1,
 // B(x, r) and F(x+1, r+1) compare the same pair (FF[x], b[x+1]) (the fused step of
-// DESIGN.md §5.1), so B bit x of row r = NOT F bit x+1 of row r+1.
-// Only the rows the backtrack reads are written: the warm-up rows 0..P-2 hold no op of
-// the 1F1B phase, so the walk stops when it reaches them (backtrack_rows) and the sweep
-// records no bits there.
-// Layout: word i of the simulation at base[i * stride] (the lanes of a warp/CTA are
-// interleaved, so 32 lanes store 64 contiguous bytes).
+// DESIGN.md §5.1), so B bit (x, r) = NOT F bit (x+1, r+1).
+// Storage (MasterBits), per lane, lanes interleaved with `stride`:
+//   cw  the F bits of the steady rows r = P..m-1 as COLUMN words: word (blk, x) holds
+//       F bit (x, 32 blk + j) in bit j, at cw[(blk (P-1) + x - 1) stride]; rows < P
+//       read as 0 (the warm-up and row P-1 record nothing: the walk ends there);
+//   rw  the cool-down rows: F word of row m+i (bit x) at rw[i stride], i = 0..P-2,
+//       then the B words, t = 0..P-1, at rw[(P-1+t) stride].
+// The column layout lets the walk jump over the rows where the critical path stays on
+// one stage (backtrack_master): one find-last-set per stage change instead of one
+// step per row.
 #pragma once
 #include "ap_device.cuh"
 
 namespace apdev {
 
-struct Bits16 {
-  uint16_t* base;  // fw[0 .. m+P-2], then bw[0 .. P-1]
+struct MasterBits {
+  uint32_t* cw;  // column words of the steady F bits
+  uint16_t* rw;  // cool-down row words (F, then B)
   int stride;
 };
+// per-lane sizes: 32-bit column words, then 16-bit row words
+__host__ __device__ inline int master_col_words(int m, int P) { return (((m - 1) >> 5) + 1) * (P - 1); }
+__host__ __device__ inline int master_row_words(int P) { return 2 * P - 1; }
+__host__ __device__ inline size_t master_bits_bytes(int m, int P, int lanes) {
+  return ((size_t)master_col_words(m, P) * 4 + (size_t)master_row_words(P) * 2) * (size_t)lanes;
+}
 
 // n = max(a, t); word += BIT if a > t.  The compare and the max are ALU instructions,
 // the bit goes in with a predicated IMAD (FMA pipe), so one decision costs two ALU
@@ -100,58 +110,94 @@ AP_DEV_INLINE void cool_row_x(uint32_t (&FF)[P], uint32_t (&L)[P], const uint32_
 }
 
 template <int P, int T>
-AP_DEV_INLINE void cool_rows(int m, uint32_t (&FF)[P], uint32_t (&L)[P], const uint32_t (&wF)[P],
-                             const uint32_t (&wB)[P], uint32_t& b, Bits16 br, uint16_t* bw,
-                             uint32_t one) {
+AP_DEV_INLINE void cool_rows(uint32_t (&FF)[P], uint32_t (&L)[P], const uint32_t (&wF)[P],
+                             const uint32_t (&wB)[P], uint32_t& b, MasterBits br, uint32_t one) {
   if constexpr (T < P) {
     uint32_t wordB = 0, wordF = 0;
     b = madd(FF[P - 1], wB[P - 1], one);
     cool_row_x<P, T, P - 2>(FF, L, wF, wB, b, wordF, wordB, one);
-    bw[(size_t)T * br.stride] = (uint16_t)wordB;
-    if constexpr (T < P - 1) br.base[(size_t)(m + T) * br.stride] = (uint16_t)wordF;
-    cool_rows<P, T + 1>(m, FF, L, wF, wB, b, br, bw, one);
+    br.rw[(size_t)(P - 1 + T) * br.stride] = (uint16_t)wordB;
+    if constexpr (T < P - 1) br.rw[(size_t)T * br.stride] = (uint16_t)wordF;
+    cool_rows<P, T + 1>(FF, L, wF, wB, b, br, one);
   }
 }
+
+// n = max(a, t); col += rb if a > t (rb: the row's bit in its column word, a register;
+// the add is a predicated IMAD on the FMA pipe, as max_bit)
+AP_DEV_INLINE uint32_t max_bitr(uint32_t a, uint32_t t, uint32_t& col, uint32_t rb, uint32_t one) {
+  uint32_t n;
+  asm("{\n\t.reg .pred p;\n\t"
+      "setp.gt.u32 p, %2, %3;\n\t"
+      "max.u32 %0, %2, %3;\n\t"
+      "@p mad.lo.u32 %1, %4, %5, %1;\n\t}"
+      : "=r"(n), "+r"(col)
+      : "r"(a), "r"(t), "r"(rb), "r"(one));
+  return n;
+}
+
+// Column words of the steady rows: bit rb of col[x] = F bit x of the current row;
+// advance() moves to the next row and stores the P-1 words when a 32-row block is full.
+template <int P>
+struct ColAcc {
+  uint32_t col[P];  // col[x], x = 1..P-1 (col[0] unused)
+  uint32_t rb;
+  uint32_t* cw;
+  int stride;
+  AP_DEV_INLINE void flush() {
+#pragma unroll
+    for (int x = 1; x < P; ++x) {
+      cw[(size_t)(x - 1) * stride] = col[x];
+      col[x] = 0;
+    }
+    cw += (size_t)(P - 1) * stride;
+  }
+  AP_DEV_INLINE void advance() {
+    rb <<= 1;
+    if (rb == 0u) {  // warp-uniform: every lane is on the same row
+      flush();
+      rb = 1u;
+    }
+  }
+};
 
 // One fused steady step in the offset form that also records the F
 // bits of the next row: n'[x] = max(n'[x+1] + s[x+1], N[x-1]), bit x+1 = N[x-1] >
 // n'[x+1] + s[x+1] (= FF[x] > b[x+1]); at x = 0 the intra operand is N[0] + s[0].
 template <int P, int X>
-AP_DEV_INLINE void nstep_bits_x(uint32_t (&n)[P], const uint32_t (&N)[P], const uint32_t (&sw)[P],
-                                uint32_t& word, uint32_t one) {
+AP_DEV_INLINE void nstep_cols_x(uint32_t (&n)[P], const uint32_t (&N)[P], const uint32_t (&sw)[P],
+                                ColAcc<P>& ca, uint32_t one) {
   if constexpr (X >= 1) {
     uint32_t t;
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(t) : "r"(n[X + 1]), "r"(one), "r"(sw[X + 1]));
-    n[X] = max_bit<(1u << (X + 1))>(N[X - 1], t, word, one);
-    nstep_bits_x<P, X - 1>(n, N, sw, word, one);
+    n[X] = max_bitr(N[X - 1], t, ca.col[X + 1], ca.rb, one);
+    nstep_cols_x<P, X - 1>(n, N, sw, ca, one);
   } else {
     uint32_t t, u;
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(t) : "r"(n[1]), "r"(one), "r"(sw[1]));
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(u) : "r"(N[0]), "r"(one), "r"(sw[0]));
-    n[0] = max_bit<2u>(u, t, word, one);
+    n[0] = max_bitr(u, t, ca.col[1], ca.rb, one);
   }
 }
 
 template <int P>
-AP_DEV_INLINE uint32_t nstep_bits(uint32_t (&N)[P], const uint32_t (&sw)[P], uint32_t one) {
+AP_DEV_INLINE void nstep_cols(uint32_t (&N)[P], const uint32_t (&sw)[P], ColAcc<P>& ca, uint32_t one) {
   static_assert(P >= 3, "");
-  uint32_t n[P], word = 0, t;
+  uint32_t n[P], t;
   asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(t) : "r"(N[P - 2]), "r"(one), "r"(sw[P - 1]));
-  n[P - 2] = max_bit<(1u << (P - 1))>(N[P - 3], t, word, one);
-  nstep_bits_x<P, P - 3>(n, N, sw, word, one);
+  n[P - 2] = max_bitr(N[P - 3], t, ca.col[P - 1], ca.rb, one);
+  nstep_cols_x<P, P - 3>(n, N, sw, ca, one);
 #pragma unroll
   for (int x = 0; x <= P - 2; ++x) N[x] = n[x];
-  return word;
 }
 
 // T (u32; >= S means "not exact, recompute") of one candidate, k = 1, p == P, m >= P,
-// with the decision words above.  wF/wB: stage weights incl. the receiver-side Comm.
+// with the decision bits above.  wF/wB: stage weights incl. the receiver-side Comm.
 // Values are clamped to S every CR rows of the steady part; the caller's S leaves room
 // for max(CR, P) + 1 rows of growth (heur_fast_bound).
 template <int P>
-AP_DEV_INLINE uint32_t sim_bits16(int m, const uint32_t (&wF)[P], const uint32_t (&wB)[P],
-                                  uint32_t S, int CR, Bits16 br, uint32_t one) {
-  static_assert(P >= 2 && P <= 16, "16-bit decision words");
+AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t (&wB)[P],
+                                  uint32_t S, int CR, MasterBits br, uint32_t one) {
+  static_assert(P >= 2 && P <= 16, "16-bit cool-down words");
   uint32_t FF[P], L[P];
   // micro-batch 0 (k = 1): F(x, 0) in row x, cross predecessor only (no bit)
   FF[0] = wF[0];
@@ -172,8 +218,14 @@ AP_DEV_INLINE uint32_t sim_bits16(int m, const uint32_t (&wF)[P], const uint32_t
   if (P >= 2) FF[0] = L[0] + wF[0];
 #pragma unroll
   for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
-  int r = P - 1;  // the row whose B part the next step computes
   int rem = m - P;
+  // the steady rows' F bits, rows P..m-1, as column words (bits of rows < P stay 0)
+  ColAcc<P> ca;
+#pragma unroll
+  for (int x = 0; x < P; ++x) ca.col[x] = 0;
+  ca.rb = 1u << P;
+  ca.cw = br.cw;
+  ca.stride = br.stride;
   if constexpr (P >= 3) {
     if (rem > 0) {
       uint32_t c[P], sw[P], N[P];
@@ -182,26 +234,22 @@ AP_DEV_INLINE uint32_t sim_bits16(int m, const uint32_t (&wF)[P], const uint32_t
       for (int x = 1; x < P; ++x) c[x] = c[x - 1] + wF[x];
 #pragma unroll
       for (int x = 0; x < P; ++x) sw[x] = wF[x] + wB[x];
-      {  // first fused step in the M-form, kept as N = M - c
-        uint32_t word = 0;
+      {  // first fused step in the M-form, kept as N = M - c (F bits of row P)
         uint32_t b = FF[P - 1] + wB[P - 1];
 #pragma unroll
         for (int x = P - 2; x >= 0; --x) {
-          word |= (FF[x] > b ? 1u : 0u) << (x + 1);
-          const uint32_t M = max(FF[x], b);
+          const uint32_t M = max_bitr(FF[x], b, ca.col[x + 1], ca.rb, one);
           N[x] = M - c[x];
           b = M + wB[x];
         }
-        br.base[(size_t)(r + 1) * br.stride] = (uint16_t)word;
-        ++r;
+        ca.advance();
       }
       int blk = (rem < CR ? rem : CR) - 1;
       rem -= blk + 1;
       for (;;) {
         for (; blk > 0; --blk) {
-          const uint32_t word = nstep_bits<P>(N, sw, one);
-          br.base[(size_t)(r + 1) * br.stride] = (uint16_t)word;
-          ++r;
+          nstep_cols<P>(N, sw, ca, one);
+          ca.advance();
         }
 #pragma unroll
         for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
@@ -220,63 +268,71 @@ AP_DEV_INLINE uint32_t sim_bits16(int m, const uint32_t (&wF)[P], const uint32_t
       rem -= blk;
       for (; blk > 0; --blk) {
         const uint32_t b = FF[1] + wB[1];
-        const uint32_t word = (FF[0] > b ? 1u : 0u) << 1;
-        const uint32_t M = max(FF[0], b);
+        const uint32_t M = max_bitr(FF[0], b, ca.col[1], ca.rb, one);
         FF[1] = M + wF[1];
         FF[0] = M + wB[0] + wF[0];
-        br.base[(size_t)(r + 1) * br.stride] = (uint16_t)word;
-        ++r;
+        ca.advance();
       }
 #pragma unroll
       for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
     }
   }
+  // the last, partial block (rb == 1: the previous row filled a block, already stored)
+  if (m > P && ca.rb != 1u) ca.flush();
   // cool-down t = 0..P-1 (row m-1+t): B of the row, F of the next row for x >= t+1.
   // Stages x < t ran their last forward already: their B reads L[x].
-  uint16_t* bw = br.base + (size_t)(m + P - 1) * br.stride;
   uint32_t b = 0;
-  cool_rows<P, 0>(m, FF, L, wF, wB, b, br, bw, one);
+  cool_rows<P, 0>(FF, L, wF, wB, b, br, one);
   return b;
 }
 
-// Master stage of the simulation recorded by sim_bits16 (same P, m): walk the unique
-// critical path back from the sink B(0, m-1) (row m+P-2) to the source F(0, 0) with
-// the tie rule of Q10, and count per stage its ops in the 1F1B phase (rows [P-1,
-// m-1+x] of stage x, for F and B alike); master = most ops, ties -> higher stage, P-1
-// if none (Q11).
-// Every edge of the path stays in its row (B(x) -> B(x+1) cross, B(x) -> F(x) intra)
-// or goes one row up (F(x) -> F(x-1) cross, F(x) -> B(x) / F(x) intra, cool-down
-// B(x) -> B(x)), so the walk runs row by row, r = m+P-2 .. 0, the same loop in every
-// lane of a warp: per row one B-chain (almost always empty), at most one B and one F
-// op.  Per-stage counts are CB-bit fields of NW registers, flushed when the path
-// changes stage.  CB = 8 needs 2m <= 255.
+// Master stage of the simulation recorded by sim_master (same P, m): walk the unique
+// critical path back from the sink B(0, m-1) (row m+P-2) to the source with the tie
+// rule of Q10, and count per stage its ops in the 1F1B phase (rows [P-1, m-1+x] of
+// stage x, for F and B alike); master = most ops, ties -> higher stage, P-1 if none
+// (Q11).  Every edge of the path stays in its row (B(x) -> B(x+1) cross, B(x) -> F(x)
+// intra) or goes one row up (F(x) -> F(x-1) cross, F(x) -> B(x) intra, cool-down
+// B(x) -> B(x)).  Per-stage counts are CB-bit fields of NW registers, flushed when the
+// path changes stage.  CB = 8 needs 2m <= 255.
+//  1. Cool-down rows m+P-2 .. m-1, one row per step, as the row words dictate.
+//  2. Steady rows m-2 .. P-1: on B(x, r) the path stays on stage x (B(x, r) -> F(x, r)
+//     -> B(x, r-1), two ops per row) until the first row r' <= r with
+//       B bit (x, r') = NOT F bit (x+1, r'+1)   (B takes B(x+1)), or  F bit (x, r'),
+//     the highest set bit of (col[x] | ~(col[x+1] >> 1)) below r: one find-last-set
+//     per stage change (or per 32-row block), not one step per row.
 template <int P, int CB>
-AP_DEV_INLINE int backtrack_rows(int m, Bits16 br) {
+AP_DEV_INLINE int backtrack_master(int m, MasterBits br) {
   constexpr unsigned PER = 32 / CB;
   constexpr int NW = (P + PER - 1) / PER;
   constexpr uint32_t maskB = (1u << (P - 1)) - 1u;  // B bits of stages 0..P-2
-  const uint16_t* fw = br.base;
-  const uint16_t* bw = br.base + (size_t)(m + P - 1) * br.stride;
+  const uint16_t* fw = br.rw;                        // F words of rows m .. m+P-2
+  const uint16_t* bw = br.rw + (size_t)(P - 1) * br.stride;
+  const uint32_t* cw = br.cw;
   const int st = br.stride;
-  uint32_t cw[NW];
+  uint32_t cnt[NW];
 #pragma unroll
-  for (int w = 0; w < NW; ++w) cw[w] = 0;
+  for (int w = 0; w < NW; ++w) cnt[w] = 0;
   auto flush = [&](unsigned x, uint32_t run) {
     const uint32_t inc = run << (CB * (x % PER));
 #pragma unroll
-    for (int w = 0; w < NW; ++w) cw[w] += (w == (int)(x / PER)) ? inc : 0u;
+    for (int w = 0; w < NW; ++w) cnt[w] += (w == (int)(x / PER)) ? inc : 0u;
+  };
+  // F bit (x, r) of a steady row r <= m-1 (stage 0 has none)
+  auto fbit = [&](unsigned x, int r) -> uint32_t {
+    return x >= 1 ? (cw[(size_t)((r >> 5) * (P - 1) + (int)x - 1) * st] >> (r & 31)) & 1u : 0u;
   };
   unsigned x = 0;
   bool onB = true;
   uint32_t run = 0, wn = 0;  // wn: F word of row r+1
-  // rows r < P-1 hold no 1F1B-phase op (warm-up forwards only): the counts are final
-  // once the walk leaves row P-1
-  for (int r = m + P - 2; r >= P - 1; --r) {
-    const uint32_t wr = fw[(size_t)r * st];
+  // 1. the cool-down rows (t = r - (m-1) = P-1 .. 0)
+  for (int r = m + P - 2; r >= m - 1; --r) {
+    const int t = r - (m - 1);
+    // F word of row r (row m-1 is a steady row: its bits are in the columns, and
+    // only the one of the stage the walk is on after its B chain is read)
+    const uint32_t wr = (t > 0) ? (uint32_t)fw[(size_t)(t - 1) * st] : 0u;
     if (onB) {
       // B bits of row r: NOT the F bits of row r+1 where stage x+1 forwards in row r+1
-      // (x >= t = r-(m-1) in the cool-down), the stored ones for x < t
-      const int t = r - (m - 1);
+      // (x >= t), the stored ones for x < t
       uint32_t bB = ~(wn >> 1) & maskB;
       if (t > 0) bB = (bB & ~((1u << t) - 1u)) | (uint32_t)bw[(size_t)t * st];
       uint32_t tt = bB >> x;  // bit j: B(x+j, r) takes its cross predecessor B(x+j+1, r)
@@ -301,25 +357,74 @@ AP_DEV_INLINE int backtrack_rows(int m, Bits16 br) {
       }
       // F(x, r) next, same row
     }
-    // F(x, r), micro-batch r - x, in the 1F1B phase (r >= P-1)
+    // F(x, r), micro-batch r - x, in the 1F1B phase
     ++run;
-    if ((wr >> x) & 1u) {  // cross: F(x-1, r-1) (x >= 1; r > x here)
+    if ((t > 0 ? (wr >> x) & 1u : fbit(x, r)) != 0u) {  // cross: F(x-1, r-1)
       flush(x, run);
       run = 0;
       --x;
       onB = false;
     } else {
-      onB = true;  // B(x, r-1), or for r = P-1 the warm-up (the loop ends)
+      onB = true;  // B(x, r-1)
     }
     wn = wr;
+  }
+  // 2. the steady rows, by column words (rows < P-1 are warm-up forwards: not counted)
+  const int lastb = (m - 1) >> 5;
+  int r = m - 2;
+  while (r >= P - 1) {
+    const int b = r >> 5, rl = r & 31;
+    const uint32_t* cb = cw + (size_t)(b * (P - 1)) * st;
+    if (onB) {
+      const uint32_t cx = x >= 1 ? cb[(size_t)(x - 1) * st] : 0u;
+      // bit j of nx: F bit (x+1, 32b + j + 1); row 32b+32 is block b+1's bit 0 (it
+      // exists whenever it can be read: j <= rl and 32b + rl + 1 <= m-1)
+      uint32_t nx = 0xffffffffu;  // stage P-1 has no cross B predecessor
+      if ((int)x <= P - 2) {
+        const uint32_t lo = cb[(size_t)x * st] >> 1;
+        const uint32_t hi = b < lastb ? cb[(size_t)((P - 1) + x) * st] << 31 : 0u;
+        nx = lo | hi;
+      }
+      const int lo_row = b == 0 ? P - 1 : 0;  // rows < P-1 are not walked
+      uint32_t E = (cx | ~nx) & ((2u << rl) - 1u) & ~((1u << lo_row) - 1u);
+      if (E == 0u) {  // stays on stage x down to the block's first walked row
+        run += 2u * (uint32_t)(rl - lo_row + 1);
+        r = 32 * b + lo_row - 1;
+        continue;
+      }
+      const int j = 31 - __clz(E);
+      run += 2u * (uint32_t)(rl - j);
+      r = 32 * b + j;
+      if ((~nx >> j) & 1u) {  // B(x, r) takes B(x+1, r)
+        flush(x, run + 1u);
+        run = 0;
+        ++x;
+      } else {  // B(x, r) -> F(x, r) -> F(x-1, r-1)
+        flush(x, run + 2u);
+        run = 0;
+        --x;
+        --r;
+        onB = false;
+      }
+    } else {  // F(x, r)
+      ++run;
+      if (x >= 1 && ((cb[(size_t)(x - 1) * st] >> rl) & 1u)) {
+        flush(x, run);
+        run = 0;
+        --x;
+      } else {
+        onB = true;
+      }
+      --r;
+    }
   }
   flush(x, run);
   constexpr uint32_t MASK = (CB == 8) ? 0xffu : 0xffffu;
   int best = P - 1;
-  uint32_t bc = (cw[(P - 1) / PER] >> (CB * ((P - 1) % PER))) & MASK;
+  uint32_t bc = (cnt[(P - 1) / PER] >> (CB * ((P - 1) % PER))) & MASK;
 #pragma unroll
   for (int xx = P - 2; xx >= 0; --xx) {
-    const uint32_t c = (cw[xx / PER] >> (CB * (xx % PER))) & MASK;
+    const uint32_t c = (cnt[xx / PER] >> (CB * (xx % PER))) & MASK;
     if (c > bc) {
       best = xx;
       bc = c;
@@ -328,6 +433,5 @@ AP_DEV_INLINE int backtrack_rows(int m, Bits16 br) {
   return best;
 }
 
-__host__ __device__ inline int bits16_words(int m, int P) { return m + 2 * P - 1; }
 
 }  // namespace apdev

@@ -1826,8 +1826,11 @@ AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
   return diff;
 }
 
+#ifndef AP_HEUR_MINB
+#define AP_HEUR_MINB 4
+#endif
 template <int P>
-__global__ void __launch_bounds__(hpool::NT, 4) k_heur_pool(HeurArgs A) {
+__global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs A) {
   using namespace hpool;
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;

@@ -7,7 +7,9 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-LIB = os.path.join(HERE, "libap.so")
+# AP_LIB_OUT / AP_NVCC_EXTRA build A/B variants (e.g. -DAP_MASTER_CHUNK=0) next to the
+# product library; the binding loads one with AP_LIB_PATH.
+LIB = os.environ.get("AP_LIB_OUT") or os.path.join(HERE, "libap.so")
 SOURCES = ["ap_kernels.cu", "ap_host.cu"]
 HEADERS = ["ap_device.cuh", "ap_launch.h", "ap_master.cuh", os.path.join("..", "..", "include", "ap.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
@@ -24,6 +26,7 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", 
 _SPLIT = os.environ.get("AP_SPLIT_COMPILE", "8")
 if _SPLIT != "0":
     FLAGS += ["--split-compile", _SPLIT]
+FLAGS += os.environ.get("AP_NVCC_EXTRA", "").split()
 
 
 def _stale() -> bool:
@@ -42,7 +45,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objs = []
     procs = []
     for src in SOURCES:
-        obj = os.path.join(CSRC, src.replace(".cu", ".o"))
+        obj = os.path.join(CSRC, src.replace(".cu", f".{os.getpid()}.o"))
         cmd = [NVCC, *ARCH, *FLAGS, "-c", os.path.join(CSRC, src), "-o", obj]
         if verbose:
             print(" ".join(cmd), file=sys.stderr)

@@ -1283,7 +1283,9 @@ __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
 // candidate it cannot finish exactly -- saturated at fastS, or T + master with k > 1
 // or m > 127 -- goes to A.redo for the generic k_eval.  A kernel of its own, so its
 // register allocation is not the generic path's.
-template <int P>
+// MASTER: T + master (A.master != nullptr) and T only are separate instances, so the
+// register allocation of one does not move with changes to the other.
+template <int P, bool MASTER>
 __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
   extern __shared__ __align__(16) unsigned char smem[];
   size_t used;
@@ -1329,7 +1331,7 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
       wB[x] = (s32Pb[c[x + 1]] - s32Pb[c[x]]) + ((x < P - 1) ? s32C[c[x + 1] - 1] : 0u);
     }
     bool done = false;
-    if (A.master == nullptr) {
+    if constexpr (!MASTER) {
       const ClampSched cs{0, A.CR, 1};
       const uint32_t t32 = sim_fast<P, uint32_t>(m, k, wF, wB, c, s32Pf, s32C, s32mk[k],
                                                  A.div1 != 0, S, cs, one);
@@ -1338,6 +1340,7 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
         done = true;
       }
     } else if (k == 1 && m <= 127) {
+      (void)c;
       const uint32_t t32 = sim_master<P>(m, wF, wB, S, A.CR, br, one);
       if (t32 < S) {
         A.time_ns[i] = (int64_t)t32;
@@ -2873,11 +2876,12 @@ static cudaError_t eval_fast_P(const EvalArgs& A, cudaStream_t s, int* launches)
   const size_t smem = ((tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15)) +
                       ((eval_fast_smem(A.t.n) + 15) & ~size_t(15)) +
                       (A.master ? master_bits_bytes(A.m, P, threads) : 0);
-  cudaError_t e = set_smem((const void*)k_eval_fast<P>, smem);
+  const void* fn = A.master ? (const void*)k_eval_fast<P, true> : (const void*)k_eval_fast<P, false>;
+  cudaError_t e = set_smem(fn, smem);
   if (e != cudaSuccess) return e;
   int occ = 0, dev = 0;
   cudaGetDevice(&dev);
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval_fast<P>, threads, smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, threads, smem);
   if (e != cudaSuccess) return e;
   occ = occ < 1 ? 1 : occ;
   int64_t blocks = (A.count + threads - 1) / threads;
@@ -2885,7 +2889,10 @@ static cudaError_t eval_fast_P(const EvalArgs& A, cudaStream_t s, int* launches)
   if (blocks > wave) blocks = wave;
   if (blocks > 0) {
     count_launch();
-    k_eval_fast<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+    if (A.master)
+      k_eval_fast<P, true><<<(unsigned)blocks, threads, smem, s>>>(A);
+    else
+      k_eval_fast<P, false><<<(unsigned)blocks, threads, smem, s>>>(A);
     if (launches) ++*launches;
   }
   return cudaGetLastError();

@@ -190,6 +190,58 @@ AP_DEV_INLINE void nstep_cols(uint32_t (&N)[P], const uint32_t (&sw)[P], ColAcc<
   for (int x = 0; x <= P - 2; ++x) N[x] = n[x];
 }
 
+// Aligned 8-row chunks of the steady rows (AP_MASTER_CHUNK, default on).  Row j of a
+// chunk that starts at a row r with r % 8 == 0 puts its bits at rbase << j, rbase = the
+// bit of row r in its column word, so every bit is a predicated IMAD with an immediate
+// multiplier and the 8 rows are one straight-line block: ptxas can overlap the rows
+// (row r+1's first decision needs only row r's second), where the one-row loop with its
+// block-full test after every row ran each row's 15-decision chain alone.  The value
+// itself is one fused add+max (VIADDMNMX) on the chain; the compare that sets the bit
+// uses its own add (t, an IMAD with the runtime `one`, so it is not merged into the
+// chain) and sits beside it.
+#ifndef AP_MASTER_CHUNK
+#define AP_MASTER_CHUNK 1
+#endif
+template <uint32_t MUL>
+AP_DEV_INLINE uint32_t dec_chunk(uint32_t nx1, uint32_t s, uint32_t a, uint32_t& col,
+                                 uint32_t rbase, uint32_t one) {
+  uint32_t t;
+  asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(t) : "r"(nx1), "r"(one), "r"(s));
+  const uint32_t n = max(nx1 + s, a);
+  asm("{\n\t.reg .pred p;\n\t"
+      "setp.gt.u32 p, %1, %2;\n\t"
+      "@p mad.lo.u32 %0, %3, %4, %0;\n\t}"
+      : "+r"(col)
+      : "r"(a), "r"(t), "r"(rbase), "n"(MUL));
+  return n;
+}
+
+template <int P, int J, int X>
+AP_DEV_INLINE void chunk_row_x(uint32_t (&n)[P], const uint32_t (&N)[P], const uint32_t (&sw)[P],
+                               uint32_t (&col)[P], uint32_t rbase, uint32_t one) {
+  if constexpr (X >= 1) {
+    n[X] = dec_chunk<(1u << J)>(n[X + 1], sw[X + 1], N[X - 1], col[X + 1], rbase, one);
+    chunk_row_x<P, J, X - 1>(n, N, sw, col, rbase, one);
+  } else {
+    uint32_t u;
+    asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(u) : "r"(N[0]), "r"(one), "r"(sw[0]));
+    n[0] = dec_chunk<(1u << J)>(n[1], sw[1], u, col[1], rbase, one);
+  }
+}
+
+template <int P, int J>
+AP_DEV_INLINE void chunk_rows(uint32_t (&N)[P], const uint32_t (&sw)[P], uint32_t (&col)[P],
+                              uint32_t rbase, uint32_t one) {
+  if constexpr (J < 8) {
+    uint32_t n[P];
+    n[P - 2] = dec_chunk<(1u << J)>(N[P - 2], sw[P - 1], N[P - 3], col[P - 1], rbase, one);
+    chunk_row_x<P, J, P - 3>(n, N, sw, col, rbase, one);
+#pragma unroll
+    for (int x = 0; x <= P - 2; ++x) N[x] = n[x];
+    chunk_rows<P, J + 1>(N, sw, col, rbase, one);
+  }
+}
+
 // T (u32; >= S means "not exact, recompute") of one candidate, k = 1, p == P, m >= P,
 // with the decision bits above.  wF/wB: stage weights incl. the receiver-side Comm.
 // Values are clamped to S every CR rows of the steady part; the caller's S leaves room
@@ -244,6 +296,37 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
         }
         ca.advance();
       }
+#if AP_MASTER_CHUNK
+      // rows P+1 .. m-1: single rows up to an 8-aligned row, aligned 8-row chunks, single
+      // rows for the rest; a clamp whenever the next piece would take the rows since the
+      // last one past CR (the caller's S leaves room for CR + 1 rows of growth)
+      int r = P + 1, since = 1;
+      const int mrow = P + rem;  // = m
+      while (r < mrow) {
+        const bool chunk = CR >= 8 && (r & 7) == 0 && r + 8 <= mrow;
+        const int len = chunk ? 8 : 1;
+        if (since + len > CR) {
+#pragma unroll
+          for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
+          since = 0;
+        }
+        if (chunk) {
+          chunk_rows<P, 0>(N, sw, ca.col, ca.rb, one);
+          ca.rb <<= 8;
+          if (ca.rb == 0u) {
+            ca.flush();
+            ca.rb = 1u;
+          }
+        } else {
+          nstep_cols<P>(N, sw, ca, one);
+          ca.advance();
+        }
+        r += len;
+        since += len;
+      }
+#pragma unroll
+      for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
+#else
       int blk = (rem < CR ? rem : CR) - 1;
       rem -= blk + 1;
       for (;;) {
@@ -257,6 +340,7 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
         blk = rem < CR ? rem : CR;
         rem -= blk;
       }
+#endif
 #pragma unroll
       for (int x = 0; x <= P - 2; ++x) FF[x + 1] = N[x] + c[x + 1];
       FF[0] = N[0] + c[0] + sw[0];

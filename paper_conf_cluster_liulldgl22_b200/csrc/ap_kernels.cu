@@ -1802,10 +1802,25 @@ constexpr int RING = 128;         // job ring per warp, >= 4 * NSW
 // Child idx (0 a, 1 a', 2 b, 3 b') of `cur` with master i (
 // reading Q17), as k_heur's gen_child, built in place in shared memory (no local
 // arrays); false if invalid or a duplicate (a' == a, b' == b).
+// Cut vectors of the warp pools are CP-padded int16 rows, 16-byte aligned, copied as
+// CP/8 16-byte words (CP = 0: element by element, p + 1 entries).
+template <int CP>
+AP_DEV_INLINE void copy_cuts(int16_t* dst, const int16_t* src, int p) {
+  if constexpr (CP > 0) {
+    static_assert(CP % 8 == 0, "");
+#pragma unroll
+    for (int q = 0; q < CP / 8; ++q)
+      reinterpret_cast<uint4*>(dst)[q] = reinterpret_cast<const uint4*>(src)[q];
+  } else {
+    for (int x = 0; x <= p; ++x) dst[x] = src[x];
+  }
+}
+
+template <int CP = 0>
 AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
                               const int16_t* s_arg, int16_t* cand) {
   if (cur[i + 1] - cur[i] < 2) return false;
-  for (int x = 0; x <= p; ++x) cand[x] = cur[x];
+  copy_cuts<CP>(cand, cur, p);
   int j, e;
   if (idx <= 1) {
     cand[i] += 1;  // first block of stage i -> stage i-1
@@ -1849,9 +1864,10 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
   // per-warp slot state: cut vectors [slot][0 cur | 1 best][P+1]; a job is a slot and a
   // code (0-3: child a, a', b, b' of cur, 4: cur itself), and the lane that simulates it
   // rebuilds the child in its own scratch vector (s_scr) from cur
-  __shared__ int16_t s_cuts[NW][NSW][2][P + 1];
+  constexpr int CP = ((P + 1 + 7) / 8) * 8;  // padded cut row (copy_cuts)
+  __shared__ __align__(16) int16_t s_cuts[NW][NSW][2][CP];
   static_assert(NSW <= 32 && 4 * NSW <= RING, "");
-  __shared__ int16_t s_scr[NW][32][P + 1];
+  __shared__ __align__(16) int16_t s_scr[NW][32][CP];
   __shared__ uint32_t s_chT[NW][NSW][4];
   __shared__ int8_t s_chM[NW][NSW][4];
   __shared__ int8_t s_curM[NW][NSW];
@@ -1900,7 +1916,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
         if (st == 1) {  // the start was simulated
           curM = s_chM[w][lane][0];
           bestT = s_chT[w][lane][0];
-          for (int x = 0; x <= P; ++x) best[x] = cur[x];
+          copy_cuts<CP>(best, cur, P);
           steps = 0;
           nsims = 1;
         } else {  // the children of a step were simulated: visit them in child order
@@ -1913,8 +1929,8 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
             const int Mc = s_chM[w][lane][idx];
             if (Tc < bestT) {
               bestT = Tc;
-              pool_child(cur, idx, curM, p, P1, s_arg, scr);
-              for (int x = 0; x <= P; ++x) best[x] = scr[x];
+              pool_child<CP>(cur, idx, curM, p, P1, s_arg, scr);
+              copy_cuts<CP>(best, scr, P);
             }
             if (Mc <= curM && Tc < selT) {
               selT = Tc;
@@ -1925,8 +1941,8 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
           if (sel < 0) {
             walk = false;  // no child qualifies
           } else {
-            pool_child(cur, sel, curM, p, P1, s_arg, scr);
-            for (int x = 0; x <= P; ++x) cur[x] = scr[x];
+            pool_child<CP>(cur, sel, curM, p, P1, s_arg, scr);
+            copy_cuts<CP>(cur, scr, P);
             curM = selM;
           }
         }
@@ -1936,7 +1952,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
         if (walk && steps < smax && curM != 0) {
           ++steps;
           for (int idx = 0; idx < 4; ++idx)
-            if (pool_child(cur, idx, curM, p, P1, s_arg, scr)) {
+            if (pool_child<CP>(cur, idx, curM, p, P1, s_arg, scr)) {
               valid |= 1 << idx;
               ++nj;
             }
@@ -2023,7 +2039,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
       const int sl = job >> 3, code = job & 7;
       const int16_t* src = s_cuts[w][sl][0];
       if (code < 4) {
-        pool_child(src, code, s_curM[w][sl], p, P1, s_arg, scr);
+        pool_child<CP>(src, code, s_curM[w][sl], p, P1, s_arg, scr);
         src = scr;
       }
       int c[P + 1];

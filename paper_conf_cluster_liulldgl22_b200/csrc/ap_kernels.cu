@@ -1798,6 +1798,15 @@ constexpr int NW = NT / 32;
 constexpr int NSW = AP_HEUR_NSW;  // restart slots per warp (lanes 0..NSW-1 own them)
 constexpr int RING = 128;         // job ring per warp, >= 4 * NSW
 }  // namespace hpool
+// Speculation in the lanes a pass leaves idle: for a walk waiting on
+// its step's children, simulate the children of child a under a guessed master of child
+// a (lower after a same-master move, same after a lower one: C5 walks alternate, 82 %
+// of steps); if the walk then moves to child a with that master, the next step's
+// results are already there and the walk takes two steps in one pass.  The walk, its
+// simulation count and its result are exactly those without speculation.
+#ifndef AP_HEUR_SPEC
+#define AP_HEUR_SPEC 1
+#endif
 
 // Child idx (0 a, 1 a', 2 b, 3 b') of `cur` with master i (
 // reading Q17), as k_heur's gen_child, built in place in shared memory (no local
@@ -1837,8 +1846,10 @@ AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
   bool diff = false;
   for (int jj = j; jj >= 2; --jj) {  // Algorithm 1 line 15 (alg1_prefix)
     const int st = s_arg[e * P1 + jj];
-    cand[jj - 1] = (int16_t)st;
+    // compare before the write: cand may be cur itself (in-place, the pool's
+    // speculative grandchildren); the prefix indices jj-1 <= j-1 are below the moved cut
     diff = diff || (st != cur[jj - 1]);
+    cand[jj - 1] = (int16_t)st;
     e = st;
   }
   return diff;
@@ -1847,6 +1858,49 @@ AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
 #ifndef AP_HEUR_MINB
 #define AP_HEUR_MINB 4
 #endif
+// One pool job: stage weights of the cut row `src`, sim_master and the master walk.
+// Returns T in the low word (>= S: saturated, no master) and the master in the high
+// word.  AP_HEUR_NOINLINE=1 makes it a real call (its own register allocation); A/B on
+// one box (profiles/r02_heur_pool_variants.md): inline 1.06-1.08 ms, call 1.07-1.53 ms
+// depending on the surrounding code, so it is inlined.
+#ifndef AP_HEUR_NOINLINE
+#define AP_HEUR_NOINLINE 0
+#endif
+// Everything is addressed through the dynamic shared-memory window (byte offsets), so
+// the callee knows its loads and stores are shared ones.
+template <int P>
+#if AP_HEUR_NOINLINE
+__device__ __noinline__
+#else
+AP_DEV_INLINE
+#endif
+unsigned long long pool_sim(uint32_t src_sh, uint32_t off32, int n, int m, uint32_t S, int CR,
+                            uint32_t off_cw, int tid, uint32_t one) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const uint32_t* s32Pf = reinterpret_cast<const uint32_t*>(smem + off32);
+  const uint32_t* s32Pb = s32Pf + (n + 1);
+  const uint32_t* s32C = s32Pb + (n + 1);
+  uint32_t* s_cw = reinterpret_cast<uint32_t*>(smem + off_cw);
+  const MasterBits br{s_cw + tid,
+                      reinterpret_cast<uint16_t*>(s_cw + (size_t)master_col_words(m, P) * hpool::NT) + tid,
+                      hpool::NT};
+  int c[P + 1];
+#pragma unroll
+  for (int x = 0; x <= P; ++x) {
+    short v;
+    asm volatile("ld.shared.s16 %0, [%1];" : "=h"(v) : "r"(src_sh + 2u * x));
+    c[x] = v;
+  }
+  uint32_t wF[P], wB[P];
+#pragma unroll
+  for (int x = 0; x < P; ++x) {
+    wF[x] = (s32Pf[c[x + 1]] - s32Pf[c[x]]) + ((x > 0) ? s32C[c[x] - 1] : 0u);
+    wB[x] = (s32Pb[c[x + 1]] - s32Pb[c[x]]) + ((x < P - 1) ? s32C[c[x + 1] - 1] : 0u);
+  }
+  const uint32_t t32 = sim_master<P>(m, wF, wB, S, CR, br, one);
+  const uint32_t M = t32 < S ? (uint32_t)backtrack_master<P, 8>(m, br) : 0u;
+  return (unsigned long long)t32 | ((unsigned long long)M << 32);
+}
 template <int P>
 __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs A) {
   using namespace hpool;
@@ -1874,6 +1928,13 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
   __shared__ int s_pend[NW][NSW];
   __shared__ int8_t s_aband[NW][NSW];
   __shared__ uint16_t s_ring[NW][2][RING];  // [0] walks past HOT steps, [1] the rest
+#if AP_HEUR_SPEC
+  // speculative grandchildren (lanes a pass leaves idle): the children of child a under
+  // a guessed master g of child a; M = -1 invalid child, -2 saturated (unusable)
+  __shared__ uint32_t s_spT[NW][NSW][4];
+  __shared__ int8_t s_spM[NW][NSW][4];
+  __shared__ int8_t s_spG[NW][NSW];
+#endif
   const int tid = threadIdx.x, lane = tid & 31, w = tid >> 5;
   for (int e = tid; e < narg; e += NT) s_arg[e] = A.arg[e];
   for (int e = tid; e < p - 1; e += NT) s_a1[e] = A.alg1[e];
@@ -1912,13 +1973,21 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
         A.redo[1 + slot] = r;
         st = 0;
       } else {
-        bool walk = true;
+        bool walk = true, again = true;
+        while (again) {
+        again = false;
+#if AP_HEUR_SPEC
+        // the speculation issued for this step is usable if child a is the move and its
+        // master is the guessed one (every grandchild simulated, none saturated)
+        bool su = false;
+#endif
         if (st == 1) {  // the start was simulated
           curM = s_chM[w][lane][0];
           bestT = s_chT[w][lane][0];
           copy_cuts<CP>(best, cur, P);
           steps = 0;
           nsims = 1;
+          valid = 1 << 6;  // no move yet: guess a lower master first
         } else {  // the children of a step were simulated: visit them in child order
           uint32_t selT = 0xffffffffu;
           int sel = -1, selM = 0;
@@ -1941,22 +2010,48 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
           if (sel < 0) {
             walk = false;  // no child qualifies
           } else {
+#if AP_HEUR_SPEC
+            if (sel == 0 && ((valid >> 5) & 1) && selM == s_spG[w][lane]) {
+              su = true;
+#pragma unroll
+              for (int idx = 0; idx < 4; ++idx) su = su && s_spM[w][lane][idx] != -2;
+            }
+#endif
             pool_child<CP>(cur, sel, curM, p, P1, s_arg, scr);
             copy_cuts<CP>(cur, scr, P);
+            valid = (selM == curM) ? (1 << 6) : 0;  // after a same-master move guess lower
             curM = selM;
           }
         }
         // next step (k_heur's begin_step with adjust_mode 0): the step cap, stop at
         // master 0, else the children of step 3
-        valid = 0;
+        valid &= 1 << 6;
         if (walk && steps < smax && curM != 0) {
           ++steps;
+#if AP_HEUR_SPEC
+          if (su) {  // this step's children were simulated speculatively: visit them now
+            for (int idx = 0; idx < 4; ++idx) {
+              const int Mi = s_spM[w][lane][idx];
+              if (Mi >= 0) {
+                valid |= 1 << idx;
+                s_chT[w][lane][idx] = s_spT[w][lane][idx];
+                s_chM[w][lane][idx] = (int8_t)Mi;
+              }
+            }
+            if (valid & 15) {
+              st = 2;
+              again = true;
+              continue;
+            }
+          } else
+#endif
           for (int idx = 0; idx < 4; ++idx)
             if (pool_child<CP>(cur, idx, curM, p, P1, s_arg, scr)) {
               valid |= 1 << idx;
               ++nj;
             }
         }
+        }  // while (again)
         if (nj > 0) {
           s_curM[w][lane] = (int8_t)curM;
           st = 2;
@@ -2029,40 +2124,93 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
     tail[0] += tot0;
     tail[1] += tot1;
     if (!__any_sync(0xffffffffu, owner && st != 0)) break;
-    __syncwarp();
-    // ---- phase B: one queued job per lane, all simulated in step
     const int nj0 = min(tail[0] - head[0], 32);
     const int nj1 = min(tail[1] - head[1], 32 - nj0);
-    if (lane < nj0 + nj1) {
+    const int nreal = nj0 + nj1;
+#if AP_HEUR_SPEC
+    // speculation: 4 idle lanes per walk waiting on a step whose child a is valid and
+    // has not been speculated on yet; walks past HOT steps first
+    const int gs = curM - ((valid >> 6) & 1);
+    const bool spc = owner && st == 2 && !((valid >> 5) & 1) && (valid & 1) && gs >= 1;
+    const unsigned hm = __ballot_sync(0xffffffffu, spc && steps >= HOT);
+    const unsigned cm = __ballot_sync(0xffffffffu, spc && steps < HOT);
+    const int nh = __popc(hm);
+    const int ncand = min((32 - nreal) >> 2, nh + __popc(cm));
+    if (spc) {
+      const unsigned lt = (1u << lane) - 1u;
+      const int rank = (steps >= HOT) ? __popc(hm & lt) : nh + __popc(cm & lt);
+      if (rank < ncand) {
+        valid |= 1 << 5;
+        s_spG[w][lane] = (int8_t)gs;
+      }
+    }
+#else
+    const int ncand = 0;
+#endif
+    __syncwarp();
+    // ---- phase B: one queued job per lane, all simulated in step
+    bool has = false, spec = false;
+    int sl = 0, ri = 0;
+    const int16_t* src = scr;
+    if (lane < nreal) {
       const int job = lane < nj0 ? s_ring[w][0][(head[0] + lane) & (RING - 1)]
                                  : s_ring[w][1][(head[1] + lane - nj0) & (RING - 1)];
-      const int sl = job >> 3, code = job & 7;
-      const int16_t* src = s_cuts[w][sl][0];
+      const int code = job & 7;
+      sl = job >> 3;
+      ri = code & 3;  // the start's result goes to index 0
+      src = s_cuts[w][sl][0];
       if (code < 4) {
         pool_child<CP>(src, code, s_curM[w][sl], p, P1, s_arg, scr);
         src = scr;
       }
-      int c[P + 1];
-#pragma unroll
-      for (int x = 0; x <= P; ++x) c[x] = src[x];
-      uint32_t wF[P], wB[P];
-#pragma unroll
-      for (int x = 0; x < P; ++x) {
-        wF[x] = (s32Pf[c[x + 1]] - s32Pf[c[x]]) + ((x > 0) ? s32C[c[x] - 1] : 0u);
-        wB[x] = (s32Pb[c[x + 1]] - s32Pb[c[x]]) + ((x < P - 1) ? s32C[c[x + 1] - 1] : 0u);
-      }
-      const uint32_t t32 = sim_master<P>(m, wF, wB, A.S, A.CR, br, one);
-      const int ri = code & 3;  // the start's result goes to index 0
-      if (t32 >= A.S) {
+      has = true;
+    }
+#if AP_HEUR_SPEC
+    else if (lane < nreal + 4 * ncand) {
+      int k = (lane - nreal) >> 2;
+      ri = (lane - nreal) & 3;
+      unsigned msk = k < nh ? hm : cm;
+      for (k = k < nh ? k : k - nh; k > 0; --k) msk &= msk - 1u;
+      sl = __ffs(msk) - 1;
+      spec = true;
+      copy_cuts<CP>(scr, s_cuts[w][sl][0], P);
+      pool_child<CP>(scr, 0, s_curM[w][sl], p, P1, s_arg, scr);  // child a (checked on issue)
+      has = pool_child<CP>(scr, ri, s_spG[w][sl], p, P1, s_arg, scr);
+      if (!has) s_spM[w][sl][ri] = -1;
+    }
+    // real and speculative lanes must simulate together: without the explicit
+    // reconvergence the two groups ran sim_master one after the other (ncu: 1.77x the
+    // warp-level executions of the row blocks)
+    __syncwarp();
+#endif
+    // the ring cursors move before the simulation (fewer registers live across it)
+    const bool real = lane < nreal;
+    head[0] += nj0;
+    head[1] += nj1;
+    if (has) {
+      const unsigned long long res =
+          pool_sim<P>((uint32_t)__cvta_generic_to_shared(src),
+                      (uint32_t)(reinterpret_cast<unsigned char*>(s32Pf) - smem), n, m, A.S, A.CR,
+                      (uint32_t)(reinterpret_cast<unsigned char*>(s_cw) - smem), tid, one);
+      const uint32_t t32 = (uint32_t)res;
+      const int8_t Mc = (int8_t)(res >> 32);
+      if (spec) {
+#if AP_HEUR_SPEC
+        if (t32 >= A.S) {
+          s_spM[w][sl][ri] = -2;  // unusable: the real job will abandon the restart
+        } else {
+          s_spT[w][sl][ri] = t32;
+          s_spM[w][sl][ri] = Mc;
+        }
+#endif
+      } else if (t32 >= A.S) {
         s_aband[w][sl] = 1;
       } else {
         s_chT[w][sl][ri] = t32;
-        s_chM[w][sl][ri] = (int8_t)backtrack_master<P, 8>(m, br);
+        s_chM[w][sl][ri] = Mc;
       }
-      atomicSub(&s_pend[w][sl], 1);
     }
-    head[0] += nj0;
-    head[1] += nj1;
+    if (real) atomicSub(&s_pend[w][sl], 1);
     __syncwarp();
   }
   if (A.sims) {

@@ -68,13 +68,15 @@ Executed opcodes (whole kernel, warp-instructions):
 ```
 
 Reading it:
-* 928 instructions per simulation; the ALU-pipe ones are VIADDMNMX (467 per simulation),
-  VIMNMX (36: warm-up and last slice piece, max-then-add), ISETP/VIADD/LOP3/IADD3 loop
-  control and successor (~50).  The floor is the 494 distinct maxima per simulation
+* {txt('r02_ncu_sweep.txt').split('instr/sim ')[1].split()[0]} instructions per simulation; the ALU-pipe ones are VIADDMNMX (467 per
+  simulation), VIMNMX (36: warm-up and last slice piece, max-then-add), ISETP/VIADD/LOP3/IADD3
+  loop control and successor (~50).  The floor is the 494 distinct maxima per simulation
   (DESIGN §5.3); the ALU pipe is {r['ncu']['alu_pipe_pct']:.0f} % busy.
-* The steady loop (block at 0x5530, 6 trips x 8 rows) is 7 VIADDMNMX + 1 IMAD per row,
-  44 % of the instructions; the fused cool-down is one VIADDMNMX per op (0x61f0).
-* Stalls are math_pipe_throttle / not_selected: the pipes, not latency.  No local memory.
+* The steady loop (the block executed 6 times per simulation, 6 trips x 8 rows) is 7
+  VIADDMNMX + 1 IMAD per row, ~45 % of the instructions; the fused cool-down is one
+  VIADDMNMX per op.
+* Stalls are math_pipe_throttle / not_selected: the pipes, not latency.  No local memory
+  in the loops (the class-A codegen of `r02_build_seed.md` keeps 104 B of stack outside them).
 """)
 
 open(os.path.join(P, "r02_ncu_heur.md"), "w").write(f"""# r02 -- ncu `--set full` of the heuristic restart kernel `k_heur_pool<16>` (C5)
@@ -94,15 +96,18 @@ Executed opcodes:
 ```
 
 Reading it (instr/sim is warp-instructions x 32 / simulations, so idle lanes count):
-* The steady loop with decision bits (two blocks, ~131 instructions per two rows: per
-  decision one add, one compare, one max and one predicated IMAD into the stage's column
-  word) runs ~45 times per simulation against 24 needed: about half the lanes of a pass are
-  idle.  C5's walks are bimodal (80 % end within 8 steps, 20 % take 21-29) and the kernel is
-  as long as ~30 dependent passes, most of them in the tail with few live walks per warp.
-* The critical-path walk is now one find-last-set per stage change on column words
-  (DESIGN §5.6), about 19 % of the instructions (round-1 form: 34 %).
-* Repacking the tail's walks into fewer warps between launches was measured slower
-  (`r02_heur_pool_variants.md`): the launch boundary is a barrier on the walks' chain.
+* The steady rows run as aligned 8-row chunks (the 506-instruction block: 120 decisions,
+  per decision one fused add+max, one add, one compare and one predicated IMAD into the
+  stage's column word), executed ~7.2 times per simulation against 5 needed, plus the
+  single rows before the first aligned row.
+* The cool-down (the ~1 090-instruction block) and the warm-up + weights block run 1.45
+  times per simulation: a pass leaves ~30 % of its lanes idle (r01/r02 before speculation:
+  ~2x); the speculating lanes (DESIGN §5.6) take part of that slack.
+* The critical-path walk is one find-last-set per stage change on column words.
+* The block at the kernel's end is the CTA's final barrier (warps that are done wait for
+  the CTA's last walk).
+* C5's walks are bimodal (80 % end within 8 steps, 20 % take 21-29), and the kernel is as
+  long as ~30 dependent passes (`r02_heur_pool_variants.md`).
 """)
 
 open(os.path.join(P, "r02_ncu_evalfast.md"), "w").write(f"""# r02 -- ncu `--set full` of `k_eval_fast<8>` with the master stage (C4, `ap_eval_batch`)

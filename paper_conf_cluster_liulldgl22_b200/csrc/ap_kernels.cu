@@ -1792,8 +1792,10 @@ __global__ void __launch_bounds__(128) k_heur(HeurArgs A) {
 namespace hpool {
 constexpr int NT = 128;   // threads per CTA (4 independent warp pools)
 constexpr int NW = NT / 32;
+// 32 slots per warp (every lane owns a walk): with speculation filling idle lanes,
+// measured 0.96-0.99 ms against 1.06-1.08 ms at 24 and 28 (profiles/r02_heur_pool_variants.md)
 #ifndef AP_HEUR_NSW
-#define AP_HEUR_NSW 24
+#define AP_HEUR_NSW 32
 #endif
 constexpr int NSW = AP_HEUR_NSW;  // restart slots per warp (lanes 0..NSW-1 own them)
 constexpr int RING = 128;         // job ring per warp, >= 4 * NSW
@@ -1958,7 +1960,10 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
   int head[2] = {0, 0}, tail[2] = {0, 0};  // warp-uniform ring cursors
   // Walks are bimodal (C5: 80 % end within 8 steps, the rest take 21-29), and the last
   // long walks set the kernel's length: the jobs of walks past HOT steps go first.
-  constexpr int HOT = 6;
+#ifndef AP_HEUR_HOT
+#define AP_HEUR_HOT 6
+#endif
+  constexpr int HOT = AP_HEUR_HOT;
   const bool owner = lane < NSW;  // lanes 0..NSW-1 own one restart slot each
   int16_t* cur = s_cuts[w][owner ? lane : 0][0];
   int16_t* best = s_cuts[w][owner ? lane : 0][1];

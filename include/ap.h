@@ -141,6 +141,19 @@ ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t
                         ap_stream_t stream);
 
 /*
+ * ap_eval_batch_ex -- ap_eval_batch that also reports how many rows were invalid (the
+ * rows it writes as time_ns = -1, master = -1: a cut vector that is not strictly
+ * increasing in [1, n-1], or k outside [1, AP_MAX_K]), so a caller can tell "some
+ * candidates were malformed" apart from a plain OK without scanning the outputs.
+ *   n_invalid  device int64 [1] or NULL; zeroed and then incremented on `stream`
+ *              (stream-ordered: read it after the stream has reached this call).
+ * Everything else as ap_eval_batch (which is ap_eval_batch_ex with n_invalid = NULL).
+ */
+ap_status ap_eval_batch_ex(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                           const int32_t* k, int64_t count, int64_t* time_ns, int32_t* master,
+                           int64_t* n_invalid, ap_stream_t stream);
+
+/*
  * ap_search_exhaustive -- exact argmin over a contiguous slice of the search space.
  * Simulates every partition with lex rank in [rank_lo, rank_hi) for every
  * k in [k_lo, k_hi] (each (partition, k) pair fully simulated, no pruning) and

@@ -73,6 +73,8 @@ def _load_lib():
     lib.ap_count.argtypes = [i32, i32, P(u64)]
     lib.ap_eval_batch.restype = i32
     lib.ap_eval_batch.argtypes = [vp, i32, i32, vp, vp, i64, vp, vp, vp]
+    lib.ap_eval_batch_ex.restype = i32
+    lib.ap_eval_batch_ex.argtypes = [vp, i32, i32, vp, vp, i64, vp, vp, vp, vp]
     lib.ap_search_exhaustive.restype = i32
     lib.ap_search_exhaustive.argtypes = [vp, i32, i32, i32, i32, u64, u64, vp, vp]
     lib.ap_search_exhaustive_mode.restype = i32
@@ -124,7 +126,7 @@ lib = _load_lib()
 # every symbol include/ap.h declares (checked by tests/test_abi.py)
 EXPORTS = ("ap_last_error", "ap_version", "ap_plan_create", "ap_plan_destroy", "ap_plan_info",
            "ap_plan_set_memory",
-           "ap_count", "ap_eval_batch", "ap_search_exhaustive", "ap_search_exhaustive_mode",
+           "ap_count", "ap_eval_batch", "ap_eval_batch_ex", "ap_search_exhaustive", "ap_search_exhaustive_mode",
            "ap_search_exhaustive2", "ap_search_exhaustive_bounded", "ap_key2_select",
            "ap_search_heuristic", "ap_search_reachable", "ap_decode_reachable",
            "ap_last_truncated",
@@ -230,14 +232,21 @@ def ap_count(n: int, p: int) -> int:
     return out.value
 
 
-def ap_eval_batch(plan: Plan, p: int, m: int, cuts, k, time_ns, master=None, stream=None):
+def ap_eval_batch(plan: Plan, p: int, m: int, cuts, k, time_ns, master=None, stream=None,
+                  n_invalid=None):
     """cuts: int32 CUDA [count, p-1]; k: int32 CUDA [count] or None; time_ns: int64
-    CUDA [count] (written); master: int32 CUDA [count] or None.  Asynchronous."""
+    CUDA [count] (written); master: int32 CUDA [count] or None; n_invalid: int64 CUDA [1]
+    or None (ap_eval_batch_ex: receives the number of invalid rows, which read -1).
+    Asynchronous."""
     count = int(time_ns.numel())
-    _check(lib.ap_eval_batch(plan.handle, int(p), int(m), _ptr(cuts, "int32", plan.device),
-                             _ptr(k, "int32", plan.device), count,
-                             _ptr(time_ns, "int64", plan.device),
-                             _ptr(master, "int32", plan.device), _stream(stream)))
+    args = (plan.handle, int(p), int(m), _ptr(cuts, "int32", plan.device),
+            _ptr(k, "int32", plan.device), count, _ptr(time_ns, "int64", plan.device),
+            _ptr(master, "int32", plan.device))
+    if n_invalid is None:
+        _check(lib.ap_eval_batch(*args, _stream(stream)))
+    else:
+        _check(lib.ap_eval_batch_ex(*args, _ptr(n_invalid, "int64", plan.device, 1),
+                                    _stream(stream)))
 
 
 def ap_search_exhaustive(plan: Plan, p: int, m: int, k_lo: int, k_hi: int, rank_lo: int,

@@ -531,19 +531,27 @@ extern "C" {
 ap_status ap_eval_batch(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
                         const int32_t* k, int64_t count, int64_t* time_ns, int32_t* master,
                         ap_stream_t stream) {
+  return ap_eval_batch_ex(plan, p, m, cuts, k, count, time_ns, master, nullptr, stream);
+}
+
+ap_status ap_eval_batch_ex(const ap_plan* plan, int32_t p, int32_t m, const int32_t* cuts,
+                           const int32_t* k, int64_t count, int64_t* time_ns, int32_t* master,
+                           int64_t* n_invalid, ap_stream_t stream) {
   g_err.clear();
   ap_status st = check_pm(plan, p, m);
   if (st != AP_OK) return st;
   if (count < 0) return fail(AP_ERR_INVALID, "count < 0");
-  if (count == 0) return AP_OK;
-  if (!time_ns || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL output/cuts");
   DeviceGuard g(plan->device);
+  if (count == 0) {
+    if (n_invalid) AP_CUDA(cudaMemsetAsync(n_invalid, 0, sizeof(*n_invalid), S_(stream)));
+    return AP_OK;
+  }
+  if (!time_ns || (p > 1 && !cuts)) return fail(AP_ERR_INVALID, "NULL output/cuts");
   int launches = 0;
-  static const int32_t kDummy = 0;
-  (void)kDummy;
   const EvalFast ef = eval_fast(plan, p);
   AP_CUDA(apk::launch_eval(plan->dev(), plan->pool, p, m, p > 1 ? cuts : nullptr, p - 1, k, 1, 0, count,
-                           time_ns, master, S_(stream), &launches, 1, 0, ef.S, ef.CR, ef.div1));
+                           time_ns, master, S_(stream), &launches, 1, 0, ef.S, ef.CR, ef.div1,
+                           reinterpret_cast<unsigned long long*>(n_invalid)));
   return AP_OK;
 }
 

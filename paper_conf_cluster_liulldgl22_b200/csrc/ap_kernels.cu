@@ -1196,6 +1196,7 @@ struct EvalArgs {
   unsigned int* redo;
   const unsigned int* redo_in;
   uint32_t one;     // = 1, opaque to the compiler (keeps the adds on IMAD)
+  unsigned long long* n_invalid;  // optional: + 1 per invalid row (zeroed by launch_eval)
 };
 // u32 copies of the prefix sums Pf, Pb, the comm and the floor(v/k) magics (fast path)
 __host__ __device__ inline size_t eval_fast_smem(int n) {
@@ -1246,6 +1247,7 @@ __global__ void __launch_bounds__(128) k_eval(EvalArgs A) {
     if (!okc || k < 1 || k > kMaxK || sl < 0 || sl > A.m) {
       A.time_ns[i] = -1;
       if (A.master) A.master[i] = -1;
+      if (A.n_invalid) atomicAdd(A.n_invalid, 1ull);
       continue;
     }
     int64_t F[P], B[P], C[P];
@@ -1322,6 +1324,7 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
     if (!okc || k < 1 || k > kMaxK) {
       A.time_ns[i] = -1;
       if (A.master) A.master[i] = -1;
+      if (A.n_invalid) atomicAdd(A.n_invalid, 1ull);
       continue;
     }
     uint32_t wF[P], wB[P];
@@ -3071,9 +3074,15 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
                         int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
                         int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches,
-                        int s_const, int s_iota, uint32_t fastS, int fastCR, int div1) {
+                        int s_const, int s_iota, uint32_t fastS, int fastCR, int div1,
+                        unsigned long long* n_invalid) {
   EvalArgs A{t, p, m, cuts, cuts_stride, kptr, k_const, k_iota, count, time_ns, master, nullptr,
-             s_const, s_iota, fastS, fastCR < 1 ? 1 : fastCR, div1, nullptr, nullptr, 1u};
+             s_const, s_iota, fastS, fastCR < 1 ? 1 : fastCR, div1, nullptr, nullptr, 1u,
+             n_invalid};
+  if (n_invalid) {
+    cudaError_t e = cudaMemsetAsync(n_invalid, 0, sizeof(*n_invalid), s);
+    if (e != cudaSuccess) return e;
+  }
   uint32_t* gbits = nullptr;
   unsigned int* redo = nullptr;
   if (fastS && count >= (1ll << 32)) fastS = A.fastS = 0;  // redo indices are 32-bit

@@ -24,13 +24,14 @@ cudaError_t launch_minlb(const DevTables& t, int p, int m, int K, int16_t* arg, 
 
 // Generic exact evaluation of `count` candidates.  cuts_stride = p-1 (batch) or 0
 // (all rows share one cut vector).  k source: kptr if non-null, else k_iota ? row+1
-// : k_const.  master may be null.  Invalid rows -> time -1, master -1.
+// : k_const.  master may be null.  Invalid rows -> time -1, master -1, and +1 on
+// *n_invalid if given (zeroed first, stream-ordered).
 cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, const int32_t* cuts,
                         int cuts_stride,
                         const int32_t* kptr, int k_const, int k_iota, int64_t count,
                         int64_t* time_ns, int32_t* master, cudaStream_t s, int* launches,
                         int s_const = 1, int s_iota = 0, uint32_t fastS = 0, int fastCR = 16,
-                        int div1 = 0);
+                        int div1 = 0, unsigned long long* n_invalid = nullptr);
 
 // Sweep parameters that depend on T_ref, computed on the device by k_sweep_prep right
 // after the T_ref evaluation and read by the sweep kernels at their start, so a search

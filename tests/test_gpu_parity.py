@@ -75,6 +75,52 @@ def test_eval_batch_invalid_rows(ap):
     assert T.cpu().tolist()[1:] == [-1, -1, -1] and T.cpu().tolist()[0] > 0
 
 
+@pytest.mark.parametrize("p,m,with_master", [(4, 8, False), (4, 8, True), (3, 8, False),
+                                             (4, 2, True)])
+def test_eval_batch_ex_counts_invalid_rows(ap, oracle_mod, p, m, with_master):
+    """ap_eval_batch_ex: the invalid-row count equals the rows written as -1, on the fast
+    kernel (p = 4, m >= p), the generic one (p = 3; m < p) and with the master; valid
+    rows still equal the oracle; a second call re-zeroes the count."""
+    import torch
+    f, b, a = synth.random_tables(7, 12)
+    plan = _plan(ap, f, b, a, synth.LINK_BYTES_PER_S)
+    M = oracle_mod.Model(f, b, a, synth.LINK_BYTES_PER_S)
+    rng = np.random.default_rng(11)
+    rows, ks, bad = [], [], []
+    for i in range(300):
+        c = sorted(rng.choice(np.arange(1, 12), p - 1, replace=False).tolist())
+        kk = int(rng.integers(1, 5))
+        kind = i % 5
+        if kind == 1:
+            c[0] = 0                      # cut outside [1, n-1]
+        elif kind == 2 and p - 1 >= 2:
+            c[0], c[1] = c[1], c[0]       # not increasing
+        elif kind == 3:
+            kk = 17                       # k > AP_MAX_K
+        rows.append(c)
+        ks.append(kk)
+        bad.append(kind in (1, 3) or (kind == 2 and p - 1 >= 2))
+    cuts = torch.tensor(rows, dtype=torch.int32, device="cuda")
+    k = torch.tensor(ks, dtype=torch.int32, device="cuda")
+    T = torch.empty(len(rows), dtype=torch.int64, device="cuda")
+    Ms = torch.empty(len(rows), dtype=torch.int32, device="cuda") if with_master else None
+    nbad = torch.full((1,), 12345, dtype=torch.int64, device="cuda")
+    for _ in range(2):
+        ap.ap_eval_batch(plan, p, m, cuts, k, T, Ms, n_invalid=nbad)
+        torch.cuda.synchronize()
+        assert int(nbad.item()) == sum(bad)
+    Th = T.cpu().tolist()
+    Mh = Ms.cpu().tolist() if with_master else None
+    for i, c in enumerate(rows):
+        if bad[i]:
+            assert Th[i] == -1 and (Mh is None or Mh[i] == -1)
+        else:
+            r = M.simulate(p, m, c, k=ks[i])
+            assert Th[i] == r["T"]
+            if Mh is not None:
+                assert Mh[i] == r["master"]
+
+
 def test_table2_partitions(ap, oracle_mod):
     """PAPER.md Table II partitions (GPT-2 345M, p=4) as named eval inputs."""
     import json

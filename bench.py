@@ -235,6 +235,26 @@ def oracle_rate(wl, budget_s: float = 10.0, runs: int = 3, threads: int = 0):
             "cpu": cpu_model()}
 
 
+def oracle_full_exhaustive(wl, runs: int = 3, threads: int = 0):
+    """The oracle's COMPLETE exhaustive search of a small config (C1, C2: BASELINE.md §4
+    'full exhaustive run, timed') on the host's cores: time to its optimal plan and
+    simulations/s, median of `runs`; its argmin is returned for comparison."""
+    import oracle
+    M = oracle.Model.from_workload(wl)
+    threads = threads or os.cpu_count() or 1
+    ts, o = [], None
+    for _ in range(runs):
+        t0 = time.perf_counter()
+        o = M.exhaustive_parallel(wl.p, wl.m, wl.k_lo, wl.k_hi, threads=threads)
+        ts.append(time.perf_counter() - t0)
+    med = statistics.median(ts)
+    return {"value": o["sims"] / med, "unit": "sims/s", "cores": threads, "kind": "oracle",
+            "time_to_optimal_plan_ms": 1e3 * med, "runs_ms": [round(1e3 * t, 2) for t in ts],
+            "T_ns": o["T"], "rank": o["rank"], "k": o["k"],
+            "sample": f"the whole search ({o['sims']} simulations), median of {runs} runs, "
+                      f"{threads} host threads", "cpu": cpu_model()}
+
+
 def oracle_heuristic_rate(wl, restarts: int = 4096, runs: int = 3, threads: int = 0):
     """The oracle's heuristic (O9) over a fixed sample of restarts [0, restarts) on the
     host's cores: simulations/s and restarts/s, median of `runs`."""
@@ -526,6 +546,12 @@ def main():
         out["cpu_baseline"] = oracle_rate(wl)
         if not args.no_secondary:
             # same-run oracle rates beside the secondary GPU numbers
+            for ci in (1, 2):
+                cb = oracle_full_exhaustive(synth.config(ci))
+                sec = out["secondary"][f"C{ci}"]
+                cb["same_plan_as_gpu"] = (cb["T_ns"], cb["rank"], cb["k"]) == \
+                    (sec["T_ns"], sec["rank"], sec["k"])
+                sec["cpu_baseline"] = cb
             out["secondary"]["C3"]["cpu_baseline"] = oracle_rate(synth.config(3), budget_s=3.0)
             out["secondary"]["C5"]["cpu_baseline"] = oracle_heuristic_rate(synth.config(5))
     if rank == 0:
@@ -537,8 +563,45 @@ def main():
 
 
 def run_secondary(ap, torch, dist, world, rank, dev, shard):
-    """C3 exhaustive and C5 heuristic (65 536 restarts + Slicer sweep), fewer steps."""
+    """C1/C2/C3 exhaustive and C5 heuristic (65 536 restarts + Slicer sweep), fewer steps."""
     out = {}
+    # C1, C2: the whole time-to-optimal-plan path (search, all-reduce, decode with critical
+    # path, Slicer sweep over the config's k range), median of 20 CUDA-event-timed runs
+    for ci in (1, 2):
+        wl = synth.config(ci)
+        f, b, a = wl.arrays()
+        plan = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=dev.index)
+        N = ap.ap_count(wl.n, wl.p)
+        lo, hi = shard(N, rank, world)
+        key = torch.empty(1, dtype=torch.int64, device=dev)
+
+        def s12():
+            if hi > lo:
+                ap.ap_search_exhaustive(plan, wl.p, wl.m, wl.k_lo, wl.k_hi, lo, hi, key)
+            else:
+                key.fill_(2 ** 63 - 1)
+            if world > 1:
+                dist.all_reduce(key, op=dist.ReduceOp.MIN)
+            res = ap.ap_decode(plan, 0, wl.p, wl.m, wl.k_lo, wl.k_hi, key=int(key.item()))
+            ap.ap_slice_sweep(plan, wl.p, wl.m, res["cuts"], max(wl.k_hi, 1))
+            return res
+        for _ in range(3):
+            s12()
+        times = []
+        for _ in range(20):
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(); r12 = s12(); e1.record(); torch.cuda.synchronize()
+            times.append(e0.elapsed_time(e1))
+        t = torch.tensor([statistics.median(times)], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        sims = N * (wl.k_hi - wl.k_lo + 1)
+        out[f"C{ci}"] = {"workload": wl.name, "sims_per_step": sims,
+                         "time_to_optimal_plan_ms": float(t[0]),
+                         "sims_per_s": sims / (float(t[0]) / 1e3), "T_ns": r12["time_ns"],
+                         "rank": r12["rank"], "k": r12["k"], "cuts": r12["cuts"],
+                         "master": r12["master"]}
     # C3
     wl = synth.config(3)
     f, b, a = wl.arrays()

@@ -98,11 +98,10 @@ Executed opcodes:
 Reading it (instr/sim is warp-instructions x 32 / simulations, so idle lanes count):
 * The steady rows run as aligned 8-row chunks (the 506-instruction block: 120 decisions,
   per decision one fused add+max, one add, one compare and one predicated IMAD into the
-  stage's column word), executed ~7.2 times per simulation against 5 needed, plus the
-  single rows before the first aligned row.
-* The cool-down (the ~1 090-instruction block) and the warm-up + weights block run 1.45
-  times per simulation: a pass leaves ~30 % of its lanes idle (r01/r02 before speculation:
-  ~2x); the speculating lanes (DESIGN §5.6) take part of that slack.
+  stage's column word), 5 per simulation, plus the single rows before the first aligned
+  row.  Per-sim execution counts above 5 (chunk) and 1 (cool-down, warm-up + weights) are
+  lanes a pass leaves idle or gives to speculation (DESIGN §5.6): ~1.3x at 32 slots per
+  warp (r02 before this session: ~2x).
 * The critical-path walk is one find-last-set per stage change on column words.
 * The block at the kernel's end is the CTA's final barrier (warps that are done wait for
   the CTA's last walk).

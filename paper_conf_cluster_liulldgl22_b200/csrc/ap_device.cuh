@@ -21,6 +21,27 @@
 
 #define AP_DEV_INLINE __device__ __forceinline__
 
+// Device-side bounds checks (AP_DEBUG_CHECKS=1 builds only; the product build compiles
+// them out).  The GPU pool refuses compute-sanitizer, so tests/test_gpu_debug_checks.py
+// builds this variant and drives every kernel family with it: a failed check prints
+// its location and traps, which fails the call.
+#ifndef AP_DEBUG_CHECKS
+#define AP_DEBUG_CHECKS 0
+#endif
+#if AP_DEBUG_CHECKS
+#include <cstdio>
+#define AP_CHECK(cond)                                                                   \
+  do {                                                                                   \
+    if (!(cond)) {                                                                       \
+      printf("AP_CHECK failed %s:%d: %s (block %d thread %d)\n", __FILE__, __LINE__,     \
+             #cond, (int)blockIdx.x, (int)threadIdx.x);                                  \
+      __trap();                                                                          \
+    }                                                                                    \
+  } while (0)
+#else
+#define AP_CHECK(cond) ((void)0)
+#endif
+
 namespace apdev {
 
 constexpr int kMaxP = 32;

@@ -686,6 +686,10 @@ __device__ __forceinline__ void sweep_range(const SweepArgs& A, uint64_t r0, uin
       }
     }
     for (uint64_t r = r0; r < r1; ++r) {
+#if AP_DEBUG_CHECKS
+      AP_CHECK(c[0] == 0 && c[P] == n);
+      for (int x = 0; x < P; ++x) AP_CHECK(c[x] < c[x + 1]);
+#endif
       // stage weights (a3): compute + receiver-side comm
       V wF[P], wB[P];
 #pragma unroll
@@ -1833,6 +1837,7 @@ AP_DEV_INLINE void copy_cuts(int16_t* dst, const int16_t* src, int p) {
 template <int CP = 0>
 AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
                               const int16_t* s_arg, int16_t* cand) {
+  AP_CHECK(i >= 0 && i < p && idx >= 0 && idx <= 3);
   if (cur[i + 1] - cur[i] < 2) return false;
   copy_cuts<CP>(cand, cur, p);
   int j, e;
@@ -1850,6 +1855,7 @@ AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
   e = cand[j];
   bool diff = false;
   for (int jj = j; jj >= 2; --jj) {  // Algorithm 1 line 15 (alg1_prefix)
+    AP_CHECK(e >= 0 && e <= cand[p]);
     const int st = s_arg[e * P1 + jj];
     // compare before the write: cand may be cur itself (in-place, the pool's
     // speculative grandchildren); the prefix indices jj-1 <= j-1 are below the moved cut
@@ -2066,9 +2072,11 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
         } else {  // the restart is finished
           my_sims += (unsigned int)nsims;
           my_key = min(my_key, ((unsigned long long)bestT << 20) | r);
-          if (A.best_out)
+          if (A.best_out) {
+            AP_CHECK(r >= A.r_lo && r < A.r_hi);
             for (int x = 1; x <= p - 1; ++x)
               A.best_out[(size_t)(r - A.r_lo) * (p - 1) + (x - 1)] = best[x];
+          }
           st = 0;
         }
       }
@@ -2131,6 +2139,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
     }
     tail[0] += tot0;
     tail[1] += tot1;
+    AP_CHECK(tail[0] - head[0] <= RING && tail[1] - head[1] <= RING);
     if (!__any_sync(0xffffffffu, owner && st != 0)) break;
     const int nj0 = min(tail[0] - head[0], 32);
     const int nj1 = min(tail[1] - head[1], 32 - nj0);
@@ -2165,6 +2174,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
                                  : s_ring[w][1][(head[1] + lane - nj0) & (RING - 1)];
       const int code = job & 7;
       sl = job >> 3;
+      AP_CHECK(sl < NSW && code <= 4);
       ri = code & 3;  // the start's result goes to index 0
       src = s_cuts[w][sl][0];
       if (code < 4) {

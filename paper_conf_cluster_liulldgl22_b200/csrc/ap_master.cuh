@@ -397,6 +397,7 @@ AP_DEV_INLINE int backtrack_master(int m, MasterBits br) {
 #pragma unroll
   for (int w = 0; w < NW; ++w) cnt[w] = 0;
   auto flush = [&](unsigned x, uint32_t run) {
+    AP_CHECK(x < (unsigned)P && run <= 2u * (uint32_t)m + 2u);
     const uint32_t inc = run << (CB * (x % PER));
 #pragma unroll
     for (int w = 0; w < NW; ++w) cnt[w] += (w == (int)(x / PER)) ? inc : 0u;
@@ -458,6 +459,7 @@ AP_DEV_INLINE int backtrack_master(int m, MasterBits br) {
   int r = m - 2;
   while (r >= P - 1) {
     const int b = r >> 5, rl = r & 31;
+    AP_CHECK(b <= ((m - 1) >> 5) && x < (unsigned)P);
     const uint32_t* cb = cw + (size_t)(b * (P - 1)) * st;
     if (onB) {
       const uint32_t cx = x >= 1 ? cb[(size_t)(x - 1) * st] : 0u;

@@ -202,9 +202,11 @@ AP_DEV_INLINE void nstep_cols(uint32_t (&N)[P], const uint32_t (&sw)[P], ColAcc<
 #ifndef AP_MASTER_CHUNK
 #define AP_MASTER_CHUNK 1
 #endif
-template <uint32_t MUL>
+// rbj = the row's bit (rbase << J, a register); the bit goes in as rbj * one with the
+// runtime `one`, which keeps it ONE predicated IMAD (with an immediate multiplier ptxas
+// folded rbase * 2^J into a hoisted register and emitted add + SEL, an ALU instruction)
 AP_DEV_INLINE uint32_t dec_chunk(uint32_t nx1, uint32_t s, uint32_t a, uint32_t& col,
-                                 uint32_t rbase, uint32_t one) {
+                                 uint32_t rbj, uint32_t one) {
   uint32_t t;
   asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(t) : "r"(nx1), "r"(one), "r"(s));
   const uint32_t n = max(nx1 + s, a);
@@ -212,20 +214,20 @@ AP_DEV_INLINE uint32_t dec_chunk(uint32_t nx1, uint32_t s, uint32_t a, uint32_t&
       "setp.gt.u32 p, %1, %2;\n\t"
       "@p mad.lo.u32 %0, %3, %4, %0;\n\t}"
       : "+r"(col)
-      : "r"(a), "r"(t), "r"(rbase), "n"(MUL));
+      : "r"(a), "r"(t), "r"(rbj), "r"(one));
   return n;
 }
 
 template <int P, int J, int X>
 AP_DEV_INLINE void chunk_row_x(uint32_t (&n)[P], const uint32_t (&N)[P], const uint32_t (&sw)[P],
-                               uint32_t (&col)[P], uint32_t rbase, uint32_t one) {
+                               uint32_t (&col)[P], uint32_t rbj, uint32_t one) {
   if constexpr (X >= 1) {
-    n[X] = dec_chunk<(1u << J)>(n[X + 1], sw[X + 1], N[X - 1], col[X + 1], rbase, one);
-    chunk_row_x<P, J, X - 1>(n, N, sw, col, rbase, one);
+    n[X] = dec_chunk(n[X + 1], sw[X + 1], N[X - 1], col[X + 1], rbj, one);
+    chunk_row_x<P, J, X - 1>(n, N, sw, col, rbj, one);
   } else {
     uint32_t u;
     asm("mad.lo.u32 %0, %1, %2, %3;" : "=r"(u) : "r"(N[0]), "r"(one), "r"(sw[0]));
-    n[0] = dec_chunk<(1u << J)>(n[1], sw[1], u, col[1], rbase, one);
+    n[0] = dec_chunk(n[1], sw[1], u, col[1], rbj, one);
   }
 }
 
@@ -233,9 +235,10 @@ template <int P, int J>
 AP_DEV_INLINE void chunk_rows(uint32_t (&N)[P], const uint32_t (&sw)[P], uint32_t (&col)[P],
                               uint32_t rbase, uint32_t one) {
   if constexpr (J < 8) {
-    uint32_t n[P];
-    n[P - 2] = dec_chunk<(1u << J)>(N[P - 2], sw[P - 1], N[P - 3], col[P - 1], rbase, one);
-    chunk_row_x<P, J, P - 3>(n, N, sw, col, rbase, one);
+    uint32_t n[P], rbj;
+    asm("mad.lo.u32 %0, %1, %2, 0;" : "=r"(rbj) : "r"(rbase), "n"(1u << J));
+    n[P - 2] = dec_chunk(N[P - 2], sw[P - 1], N[P - 3], col[P - 1], rbj, one);
+    chunk_row_x<P, J, P - 3>(n, N, sw, col, rbj, one);
 #pragma unroll
     for (int x = 0; x <= P - 2; ++x) N[x] = n[x];
     chunk_rows<P, J + 1>(N, sw, col, rbase, one);

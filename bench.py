@@ -497,6 +497,27 @@ def main():
     achieved = my_ops / k_avg_s if k_avg_s > 0 else 0.0
     clk_mhz = clk.get("sm_mhz") or sm_max
     peak, per_clk, peak_src = int_peak(clk_mhz, sms)
+    # the same roofline for the secondary kernels (achieved algorithmic int32 ops / time)
+    def sec_roof(kernel, sims, p_, m_, ks, ms):
+        if not ms or ms <= 0:
+            return None
+        ops = sims * statistics.mean(ops_per_sim(p_, m_, k) for k in ks)
+        naive = sims * statistics.mean(ops_per_sim_naive(p_, m_, k) for k in ks)
+        a = ops / (ms / 1e3)
+        return {"bound": "alu", "kernel": kernel, "achieved": a / 1e12, "peak": peak / 1e12,
+                "unit": "Tops/s (int32)", "frac": a / peak,
+                "frac_naive_count": naive / (ms / 1e3) / peak, "time_ms": ms}
+    if secondary.get("C5"):
+        c5 = secondary["C5"]
+        c5["roofline"] = sec_roof("k_heur_pool<16> (restart kernel)", c5["sims_per_step"] / max(world, 1),
+                                  16, 64, [1], c5.get("kernel_ms"))
+    if secondary.get("eval_batch"):
+        evb = secondary["eval_batch"]
+        w4 = synth.config(4)
+        for name, ks in (("T", range(w4.k_lo, w4.k_hi + 1)), ("T_master_k1", [1])):
+            if name in evb:
+                evb[name]["roofline"] = sec_roof("k_eval_fast<8> (+ exact redo pass)", 1 << 22, w4.p, w4.m,
+                                                 list(ks), evb[name]["ms"])
     roof = {"bound": "alu", "kernel": "k_sweep_exact<%d,%s>" % (wl.p, "u32" if info["fast_u32"] else "u64"),
             "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s (int32)",
             "frac": achieved / peak, "traffic": None,
@@ -660,11 +681,15 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
     plan5 = ap.ap_plan_create(f, b, a, wl.link_bytes_per_s, device=dev.index)
     rlo, rhi = shard(wl.restarts, rank, world)
 
+    k5 = []  # the restart kernel's own CUDA-event time (library events, launching stream)
+
     def s5():
         ap.ap_search_heuristic(plan5, wl.p, wl.m, wl.seed, wl.radius, rlo, rhi, 0, key)
         if world > 1:
             dist.all_reduce(key, op=dist.ReduceOp.MIN)
-        res = ap.ap_decode(plan5, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=int(key.item()))
+        kv = int(key.item())  # the step's one host read of the key (decode needs it)
+        k5.append(ap.ap_last_kernel_ms())
+        res = ap.ap_decode(plan5, 1, wl.p, wl.m, seed=wl.seed, radius=wl.radius, key=kv)
         Tk, bk = ap.ap_slice_sweep(plan5, wl.p, wl.m, res["cuts"], wl.slice_k_max)
         return res, Tk, bk
     s5()
@@ -686,7 +711,8 @@ def run_secondary(ap, torch, dist, world, rank, dev, shard):
                  "sims_per_step": int(sims5[0]),
                  "sims_per_s": float(sims5[0]) / (float(t[0]) / 1e3),
                  "time_to_plan_ms": float(t[0]), "T_ns": r5["time_ns"], "restart": r5["restart"],
-                 "cuts": r5["cuts"], "slicer_T_ns": [int(x) for x in Tk], "slicer_best_k": bk}
+                 "cuts": r5["cuts"], "slicer_T_ns": [int(x) for x in Tk], "slicer_best_k": bk,
+                 "kernel_ms": statistics.median(k5[1:]) if len(k5) > 1 else None}
     # certified bound (NEXT N3): T* >= minLB, so the plan is within `certified_gap` of optimal
     lb, _ = ap.ap_min_lower_bound(plan5, wl.p, wl.m, 1)
     out["C5"]["certified_minlb_ns"] = lb

@@ -1359,6 +1359,65 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
   }
 }
 
+// Exact pass over the candidates k_eval_fast listed as saturated (T >= its u32 bound),
+// T only, p == P, m >= P, s = 1: the same offset-form sweep in 64-bit (sim_fast<P, u64>,
+// the sweep kernels' exact variant) instead of the generic event-order kernel.  The list
+// is short (C4 random partitions: ~2 %), so the pass is one simulation per thread and
+// its length is one simulation's latency: C4 2^22 candidates, 98 us with the generic
+// kernel (profiles/r02_eval_redo.md).
+static cudaError_t set_smem(const void* fn, size_t bytes);
+int num_sms(int device);
+
+template <int P>
+__global__ void __launch_bounds__(128) k_eval_redo64(EvalArgs A) {
+  if (A.redo_in[0] == 0u) return;
+  extern __shared__ __align__(16) unsigned char smem[];
+  size_t used;
+  const Tables T = stage_and_scan(A.t.tab, A.t.n, A.t.npad, smem, &used);
+  const int n = A.t.n, m = A.m;
+  const uint64_t* sPf = reinterpret_cast<const uint64_t*>(T.Pf);
+  const uint64_t* sPb = reinterpret_cast<const uint64_t*>(T.Pb);
+  const uint64_t* sC = reinterpret_cast<const uint64_t*>(T.comm);
+  const int64_t cnt = (int64_t)A.redo_in[0];
+  const ClampSched cs{0, 1, 0};  // ignored by the 64-bit sweep
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < cnt;
+       j += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = (int64_t)A.redo_in[1 + j];
+    int c[P + 1];
+    load_cuts<P>(A.cuts + (size_t)i * A.cuts_stride, P, n, c);  // valid: checked by the fast pass
+    const int k = A.kptr ? A.kptr[i] : (A.k_iota ? (int)(i + 1) : A.k_const);
+    uint64_t wF[P], wB[P];
+#pragma unroll
+    for (int x = 0; x < P; ++x) {
+      wF[x] = (sPf[c[x + 1]] - sPf[c[x]]) + ((x > 0) ? sC[c[x] - 1] : 0ull);
+      wB[x] = (sPb[c[x + 1]] - sPb[c[x]]) + ((x < P - 1) ? sC[c[x + 1] - 1] : 0ull);
+    }
+    A.time_ns[i] = (int64_t)sim_fast<P, uint64_t>(m, k, wF, wB, c, sPf, sC, 0u, false, 0ull, cs, 1u);
+  }
+}
+
+template <int P>
+static cudaError_t eval_redo64_P(const EvalArgs& A, cudaStream_t s, int* launches) {
+  const int threads = 128;
+  const size_t smem = (tables_smem_bytes(A.t.npad, A.t.n) + 15) & ~size_t(15);
+  cudaError_t e = set_smem((const void*)k_eval_redo64<P>, smem);
+  if (e != cudaSuccess) return e;
+  int occ = 0, dev = 0;
+  cudaGetDevice(&dev);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_eval_redo64<P>, threads, smem);
+  if (e != cudaSuccess) return e;
+  occ = occ < 1 ? 1 : occ;
+  int64_t blocks = (A.count + threads - 1) / threads;
+  const int64_t wave = (int64_t)num_sms(dev) * occ;
+  if (blocks > wave) blocks = wave;
+  if (blocks > 0) {
+    count_launch();
+    k_eval_redo64<P><<<(unsigned)blocks, threads, smem, s>>>(A);
+    if (launches) ++*launches;
+  }
+  return cudaGetLastError();
+}
+
 // ===========================================================================
 // Algorithm 1, one CTA.  time[0][0] = 0, others +inf;
 // time[i][j] = min_k max(time[k][j-1], P[i]-P[k]) over k ascending, strict '<'
@@ -3146,7 +3205,19 @@ cudaError_t launch_eval(const DevTables& t, cudaMemPool_t pool, int p, int m, co
     X.fastS = 0;
     X.redo = nullptr;
     X.redo_in = redo;
-    e = run(X);
+#ifndef AP_EVAL_REDO64
+#define AP_EVAL_REDO64 1
+#endif
+    if (AP_EVAL_REDO64 && !master) {  // T only: the 64-bit offset-form sweep
+      switch (p) {
+        case 2: e = eval_redo64_P<2>(X, s, launches); break;
+        case 4: e = eval_redo64_P<4>(X, s, launches); break;
+        case 8: e = eval_redo64_P<8>(X, s, launches); break;
+        default: e = eval_redo64_P<16>(X, s, launches); break;
+      }
+    } else {
+      e = run(X);
+    }
   }
   if (gbits) cudaFreeAsync(gbits, s);
   if (redo) cudaFreeAsync(redo, s);

@@ -1347,10 +1347,14 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
         done = true;
       }
     } else if (k == 1 && m <= 127) {
+      // renormalised instead of clamped (Renorm, ap_master.cuh): exact for every
+      // candidate whose state spread stays below S, however large T is, so the
+      // saturated ones need no generic int64 pass
       (void)c;
-      const uint32_t t32 = sim_master<P>(m, wF, wB, S, A.CR, br, one);
-      if (t32 < S) {
-        A.time_ns[i] = (int64_t)t32;
+      Renorm rn;
+      const uint32_t t32 = sim_master<P, true>(m, wF, wB, S, A.CR, br, one, &rn);
+      if (rn.exact) {
+        A.time_ns[i] = (int64_t)(rn.base + t32);
         A.master[i] = backtrack_master<P, 8>(m, br);
         done = true;
       }

@@ -245,13 +245,48 @@ AP_DEV_INLINE void chunk_rows(uint32_t (&N)[P], const uint32_t (&sw)[P], uint32_
   }
 }
 
+// Every CR rows the steady state is either clamped to S (RENORM = false: a candidate
+// whose T reaches S is not exact and is recomputed by the caller) or RENORMALISED
+// (RENORM = true): the least running value is subtracted from all of them and added to
+// a 64-bit base.  The row recurrence only adds weights to state values and takes
+// maxima of them, so shifting the whole state by a constant shifts every later value by
+// it and leaves every comparison -- every decision bit -- unchanged; T = base + the
+// returned value.  The state stays within S of its minimum except in pathological
+// cases, which clear `exact` (the caller recomputes those).  Offset form: N >= 0 holds
+// after a shift by min N.
+struct Renorm {
+  unsigned long long base = 0;
+  bool exact = true;
+};
+template <int P, bool RENORM, int CNT>
+AP_DEV_INLINE void fix_state(uint32_t (&V)[P], uint32_t S, Renorm& rn) {
+  if constexpr (RENORM) {
+    uint32_t mn = V[0], mx = V[0];
+#pragma unroll
+    for (int x = 1; x < CNT; ++x) {
+      mn = min(mn, V[x]);
+      mx = max(mx, V[x]);
+    }
+#pragma unroll
+    for (int x = 0; x < CNT; ++x) V[x] -= mn;
+    rn.base += mn;
+    rn.exact = rn.exact && (mx - mn < S);
+  } else {
+#pragma unroll
+    for (int x = 0; x < CNT; ++x) V[x] = min(V[x], S);
+  }
+}
+
 // T (u32; >= S means "not exact, recompute") of one candidate, k = 1, p == P, m >= P,
 // with the decision bits above.  wF/wB: stage weights incl. the receiver-side Comm.
-// Values are clamped to S every CR rows of the steady part; the caller's S leaves room
-// for max(CR, P) + 1 rows of growth (heur_fast_bound).
-template <int P>
+// Values are clamped to S (or renormalised, see Renorm) every CR rows of the steady
+// part; the caller's S leaves room for max(CR, P) + 1 rows of growth
+// (heur_fast_bound).
+template <int P, bool RENORM = false>
 AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t (&wB)[P],
-                                  uint32_t S, int CR, MasterBits br, uint32_t one) {
+                                  uint32_t S, int CR, MasterBits br, uint32_t one,
+                                  Renorm* rnp = nullptr) {
+  Renorm rn;
   static_assert(P >= 2 && P <= 16, "16-bit cool-down words");
   uint32_t FF[P], L[P];
   // micro-batch 0 (k = 1): F(x, 0) in row x, cross predecessor only (no bit)
@@ -271,8 +306,11 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
 #pragma unroll
   for (int x = P - 2; x >= 1; --x) FF[x] = max(FF[x - 1], L[x]) + wF[x];
   if (P >= 2) FF[0] = L[0] + wF[0];
+  if constexpr (!RENORM) {  // (RENORM: the warm-up values are small, and a shift here
+                            // would break the offset form's N >= 0)
 #pragma unroll
-  for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
+    for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
+  }
   int rem = m - P;
   // the steady rows' F bits, rows P..m-1, as column words (bits of rows < P stay 0)
   ColAcc<P> ca;
@@ -309,8 +347,7 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
         const bool chunk = CR >= 8 && (r & 7) == 0 && r + 8 <= mrow;
         const int len = chunk ? 8 : 1;
         if (since + len > CR) {
-#pragma unroll
-          for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
+          fix_state<P, RENORM, P - 1>(N, S, rn);
           since = 0;
         }
         if (chunk) {
@@ -327,8 +364,7 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
         r += len;
         since += len;
       }
-#pragma unroll
-      for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
+      fix_state<P, RENORM, P - 1>(N, S, rn);
 #else
       int blk = (rem < CR ? rem : CR) - 1;
       rem -= blk + 1;
@@ -337,8 +373,7 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
           nstep_cols<P>(N, sw, ca, one);
           ca.advance();
         }
-#pragma unroll
-        for (int x = 0; x <= P - 2; ++x) N[x] = min(N[x], S);
+        fix_state<P, RENORM, P - 1>(N, S, rn);
         if (rem <= 0) break;
         blk = rem < CR ? rem : CR;
         rem -= blk;
@@ -360,8 +395,7 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
         FF[0] = M + wB[0] + wF[0];
         ca.advance();
       }
-#pragma unroll
-      for (int x = 0; x < P; ++x) FF[x] = min(FF[x], S);
+      fix_state<P, RENORM, P>(FF, S, rn);
     }
   }
   // the last, partial block (rb == 1: the previous row filled a block, already stored)
@@ -370,6 +404,7 @@ AP_DEV_INLINE uint32_t sim_master(int m, const uint32_t (&wF)[P], const uint32_t
   // Stages x < t ran their last forward already: their B reads L[x].
   uint32_t b = 0;
   cool_rows<P, 0>(FF, L, wF, wB, b, br, one);
+  if (rnp) *rnp = rn;
   return b;
 }
 

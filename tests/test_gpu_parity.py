@@ -1144,3 +1144,30 @@ def test_exhaustive_bounded(ap, oracle_mod):
         assert out.tolist() == [2**63 - 1, 2**63 - 1]
     with pytest.raises(ap.APError):
         ap.ap_search_exhaustive_bounded(plan, p, m, 1, 2, 0, N, 2, -1, out)
+
+
+def test_eval_master_renormalised_beyond_u32(ap, oracle_mod):
+    """ap_eval_batch T + master on the u32 fast path renormalises its state instead of
+    clamping it (Renorm, ap_master.cuh): candidates whose T exceeds 2^32 (C4's most
+    unbalanced partitions) are still exact, T and master equal to the oracle's."""
+    import torch
+    wl = synth.config(4)
+    f, b, a = wl.arrays()
+    plan = _plan(ap, f, b, a, wl.link_bytes_per_s)
+    M = oracle_mod.Model.from_workload(wl)
+    n, p, m = wl.n, wl.p, 100  # m = 100: the most unbalanced partitions pass 2^32 ns
+    rows = [list(range(1, p)), list(range(n - p + 1, n)), [1, 2, 3, 4, 5, 6, 40],
+            [20, 21, 22, 23, 24, 25, 26], [1, 30, 31, 32, 33, 34, 35]]
+    rng = np.random.default_rng(5)
+    while len(rows) < 64:
+        rows.append(sorted(rng.choice(np.arange(1, n), p - 1, replace=False).tolist()))
+    want = [M.simulate(p, m, r) for r in rows]
+    assert sum(w["T"] >= 2 ** 32 for w in want) >= 3
+    cuts = torch.tensor(rows, dtype=torch.int32, device="cuda")
+    k1 = torch.ones(len(rows), dtype=torch.int32, device="cuda")
+    T = torch.empty(len(rows), dtype=torch.int64, device="cuda")
+    Ms = torch.empty(len(rows), dtype=torch.int32, device="cuda")
+    ap.ap_eval_batch(plan, p, m, cuts, k1, T, Ms)
+    torch.cuda.synchronize()
+    assert T.tolist() == [w["T"] for w in want]
+    assert Ms.tolist() == [w["master"] for w in want]

@@ -156,6 +156,9 @@ AP_DEV_INLINE void clamp_n(V (&N)[P], V S) {
 #ifndef AP_NFORM
 #define AP_NFORM 1
 #endif
+#ifndef AP_EVAL_RENORM
+#define AP_EVAL_RENORM 1
+#endif
 
 template <int P, typename V>
 AP_DEV_INLINE void clamp_ff(V (&FF)[P], V S) {
@@ -231,9 +234,13 @@ struct ClampSched {
 //        G[x] = B'(x, m-2) for x <= P-2 (longest path from the end of F(x,0) via
 //               F(x,1)),   G[P-1] = F'(P-1, m-1) (via B(P-1,0)),
 //      so that T(k) = max_x (FF_x(k) + G[x]) for every k.
-template <int P, typename V, bool REV, typename CS>
+// RENORM (u32, ap_eval_batch T only): the saturating clamps become renormalisations
+// (Renorm, ap_master.cuh): the least running value moves into rn->base, so a
+// candidate past the u32 bound stays exact; the clamp right after the warm-up is
+// skipped (a shift there would break the offset form's N >= 0; those values are small).
+template <int P, typename V, bool REV, typename CS, bool RENORM = false>
 AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P], V S,
-                           CS cs, uint32_t one, V (&G)[P]) {
+                           CS cs, uint32_t one, V (&G)[P], Renorm* rn = nullptr) {
   using O = XOps<V>;
   V L[P];
   // warm-up rows r = 1..P-2: stage x <= r-1 does F(x, r-x); L == FF here
@@ -255,7 +262,7 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
     constexpr int U = (P <= 8) ? 8 : 4;
     const V wBF0 = wB[0] + wF[0];
     int rem = m - P;
-    if (sizeof(V) == 4 && cs.first() == 0) clamp_ff<P, V>(FF, S);
+    if (sizeof(V) == 4 && cs.first() == 0 && !RENORM) clamp_ff<P, V>(FF, S);
     int seg = (sizeof(V) == 4 && cs.first() > 0) ? cs.first() : cs.every();
     if (sizeof(V) != 4) seg = rem;
     if constexpr (P >= 3 && AP_NFORM) {
@@ -295,13 +302,17 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
             default: break;
           }
           if (rem <= 0) break;
-          clamp_n<P, V>(N, S);
+          if constexpr (RENORM) fix_state<P, true, P - 1>(N, S, *rn);
+          else clamp_n<P, V>(N, S);
           blk = rem < cs.every() ? rem : cs.every();
           rem -= blk;
         }
         // back to finishes (u32: FF = N + c sits up to one row's growth above N, which
         // the host's clamp_final test allows for: last segment + 1 + p rows)
-        if (cs.fin()) clamp_n<P, V>(N, S);
+        if (cs.fin()) {
+          if constexpr (RENORM) fix_state<P, true, P - 1>(N, S, *rn);
+          else clamp_n<P, V>(N, S);
+        }
 #pragma unroll
         for (int x = 0; x <= P - 2; ++x) FF[x + 1] = fma_add(N[x], c[x + 1], one);
         FF[0] = fma_add(N[0], fma_add(c[0], sw[0], one), one);
@@ -316,10 +327,13 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
         for (int u = 0; u < U; ++u) mstep<P, V>(FF, wF, wB, wBF0, one);
       }
       for (; blk > 0; --blk) mstep<P, V>(FF, wF, wB, wBF0, one);
-      if (rem > 0 || cs.fin()) clamp_ff<P, V>(FF, S);
+      if (rem > 0 || cs.fin()) {
+        if constexpr (RENORM) fix_state<P, true, P>(FF, S, *rn);  // M-form: no offsets
+        else clamp_ff<P, V>(FF, S);
+      }
       seg = cs.every();
     }
-    if (m == P && cs.fin() && cs.first() != 0) clamp_ff<P, V>(FF, S);
+    if (m == P && cs.fin() && cs.first() != 0 && !RENORM) clamp_ff<P, V>(FF, S);
   }
   // cool-down, fused the same way: step t = 0..P-1 is the backward pass of row
   // r = m-1+t plus the forward pass of row r+1, which only stages x >= t+1 still
@@ -359,6 +373,19 @@ AP_DEV_INLINE V sweep_tail(int m, V (&FF)[P], const V (&wF)[P], const V (&wB)[P]
     G[P - 1] = FF[P - 1];
   }
   return b;
+}
+
+// ap_eval_batch T only: the same with renormalisation instead of the clamps (u32);
+// T = rn.base + the returned value when rn.exact.
+template <int P>
+AP_DEV_INLINE uint32_t sim_fast_rn(int m, int k, const uint32_t (&wF)[P], const uint32_t (&wB)[P],
+                                   const int (&c)[P + 1], const uint32_t* sPf, const uint32_t* sC,
+                                   uint32_t Mk, bool div1, uint32_t S, int CR, uint32_t one,
+                                   Renorm& rn) {
+  uint32_t FF[P], G[P];
+  pieces<P, uint32_t>(k, wF, c, sPf, sC, Mk, div1, one, FF);
+  const ClampSched cs{0, CR, 1};
+  return sweep_tail<P, uint32_t, false, ClampSched, true>(m, FF, wF, wB, S, cs, one, G, &rn);
 }
 
 // Simulate one (candidate, k) for p == P, m >= P.  Returns T (u32: saturated at S).
@@ -1339,6 +1366,15 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
     }
     bool done = false;
     if constexpr (!MASTER) {
+#if AP_EVAL_RENORM
+      Renorm rn;
+      const uint32_t t32 = sim_fast_rn<P>(m, k, wF, wB, c, s32Pf, s32C, s32mk[k], A.div1 != 0, S,
+                                          A.CR, one, rn);
+      if (rn.exact) {
+        A.time_ns[i] = (int64_t)(rn.base + t32);
+        done = true;
+      }
+#else
       const ClampSched cs{0, A.CR, 1};
       const uint32_t t32 = sim_fast<P, uint32_t>(m, k, wF, wB, c, s32Pf, s32C, s32mk[k],
                                                  A.div1 != 0, S, cs, one);
@@ -1346,6 +1382,7 @@ __global__ void __launch_bounds__(128) k_eval_fast(EvalArgs A) {
         A.time_ns[i] = (int64_t)t32;
         done = true;
       }
+#endif
     } else if (k == 1 && m <= 127) {
       // renormalised instead of clamped (Renorm, ap_master.cuh): exact for every
       // candidate whose state spread stays below S, however large T is, so the

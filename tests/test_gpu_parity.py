@@ -1147,9 +1147,10 @@ def test_exhaustive_bounded(ap, oracle_mod):
 
 
 def test_eval_master_renormalised_beyond_u32(ap, oracle_mod):
-    """ap_eval_batch T + master on the u32 fast path renormalises its state instead of
-    clamping it (Renorm, ap_master.cuh): candidates whose T exceeds 2^32 (C4's most
-    unbalanced partitions) are still exact, T and master equal to the oracle's."""
+    """ap_eval_batch on the u32 fast path renormalises its state instead of clamping it
+    (Renorm, ap_master.cuh), T + master and T only: candidates whose T exceeds 2^32
+    (C4's most unbalanced partitions at m = 100) are still exact, T and master equal to
+    the oracle's."""
     import torch
     wl = synth.config(4)
     f, b, a = wl.arrays()
@@ -1171,3 +1172,10 @@ def test_eval_master_renormalised_beyond_u32(ap, oracle_mod):
     torch.cuda.synchronize()
     assert T.tolist() == [w["T"] for w in want]
     assert Ms.tolist() == [w["master"] for w in want]
+    # T only, k = 1..8: the offset-form sweep renormalises too (sim_fast_rn)
+    ks = [1 + (i % 8) for i in range(len(rows))]
+    wantk = [M.simulate(p, m, r, k=kk)["T"] for r, kk in zip(rows, ks)]
+    assert sum(t >= 2 ** 32 for t in wantk) >= 3
+    ap.ap_eval_batch(plan, p, m, cuts, torch.tensor(ks, dtype=torch.int32, device="cuda"), T)
+    torch.cuda.synchronize()
+    assert T.tolist() == wantk

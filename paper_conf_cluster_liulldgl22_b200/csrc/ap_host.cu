@@ -89,6 +89,7 @@ struct HeurCache {
   int16_t* d_best = nullptr;
   size_t cap = 0;
   bool valid = false;
+  cudaEvent_t done = nullptr;  // recorded after the search that filled d_best (its device)
 };
 thread_local HeurCache g_hcache;
 
@@ -892,6 +893,10 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   if (g_hcache.dev != plan->device || g_hcache.cap < need) {
     // stream-ordered (no device-wide synchronisation inside the search)
     if (g_hcache.d_best && g_hcache.dev == plan->device) cudaFreeAsync(g_hcache.d_best, s);
+    if (g_hcache.done && g_hcache.dev != plan->device) {
+      cudaEventDestroy(g_hcache.done);  // an event belongs to the device it was made on
+      g_hcache.done = nullptr;
+    }
     g_hcache.d_best = nullptr;
     g_hcache.cap = 0;
     AP_CUDA(cudaMallocFromPoolAsync((void**)&g_hcache.d_best, need, plan->pool, s));
@@ -913,6 +918,9 @@ ap_status ap_search_heuristic(const ap_plan* plan, int32_t p, int32_t m, uint64_
   g_hcache.r_lo = r_lo;
   g_hcache.r_hi = r_hi;
   g_hcache.adjust_mode = adjust_mode;
+  if (g_hcache.done == nullptr)  // g_hcache.dev == plan->device here (the buffer's device)
+    AP_CUDA(cudaEventCreateWithFlags(&g_hcache.done, cudaEventDisableTiming));
+  AP_CUDA(cudaEventRecord(g_hcache.done, s));
   g_hcache.valid = true;
   AP_CUDA(g_timer.record(1, s, plan->device));
   g_timer.sims_on_device = true;
@@ -1133,16 +1141,12 @@ ap_status ap_decode(const ap_plan* plan, int32_t mode, int32_t p, int32_t m, int
                           g_hcache.radius == radius && r >= g_hcache.r_lo &&
                           r < g_hcache.r_hi && g_hcache.dev == plan->device && p > 1;
       if (res == AP_OK && cached) {
-        // the search kernel already wrote restart r's best cuts: wait for it, copy them
-        int16_t h16[32];
-        e = cudaEventSynchronize(g_timer.ev[1]);
+        // the search kernel already wrote restart r's best cuts: order this stream after
+        // it and widen them to int32 on the device (no host round trip)
+        e = cudaStreamWaitEvent(s, g_hcache.done, 0);
         if (e == cudaSuccess)
-          e = cudaMemcpy(h16, g_hcache.d_best + (size_t)(r - g_hcache.r_lo) * (p - 1),
-                         2 * (size_t)(p - 1), cudaMemcpyDeviceToHost);
-        int32_t h32[32];
-        for (int x = 0; x < p - 1; ++x) h32[x] = h16[x];
-        if (e == cudaSuccess)
-          e = cudaMemcpyAsync(d_cuts, h32, 4 * (size_t)(p - 1), cudaMemcpyHostToDevice, s);
+          e = apk::launch_widen16(g_hcache.d_best + (size_t)(r - g_hcache.r_lo) * (p - 1), d_cuts,
+                                  p - 1, s);
         if (e != cudaSuccess) res = fail(AP_ERR_CUDA, "decode cache: %s", cudaGetErrorString(e));
       } else if (res == AP_OK) res = run_alg1(plan, p, sc, &d_arg, &d_a1, &d_val);
       if (res == AP_OK && !cached) {

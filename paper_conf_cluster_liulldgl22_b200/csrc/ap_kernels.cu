@@ -3760,6 +3760,15 @@ cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t*
   }
 }
 
+__global__ void k_widen16(const int16_t* src, int32_t* dst, int n) {
+  for (int i = threadIdx.x; i < n; i += blockDim.x) dst[i] = src[i];
+}
+cudaError_t launch_widen16(const int16_t* src, int32_t* dst, int n, cudaStream_t s) {
+  count_launch();
+  k_widen16<<<1, 32, 0, s>>>(src, dst, n);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s) {
   count_launch();
   k_init_key<<<1, 1, 0, s>>>(key);

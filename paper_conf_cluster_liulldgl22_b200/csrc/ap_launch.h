@@ -124,6 +124,8 @@ cudaError_t launch_cpath(const DevTables& t, int p, int m, int k, const int32_t*
 
 // key = INT64_MAX (and counter[0..2] = 0 if non-null); precedes launch_sweep/heuristic.
 cudaError_t launch_init_key(unsigned long long* key, unsigned int* counter, cudaStream_t s);
+// dst[i] = src[i] for i < n (int16 -> int32), one warp
+cudaError_t launch_widen16(const int16_t* src, int32_t* dst, int n, cudaStream_t s);
 
 // Reachable-set search (NEXT N1): restarts [r_lo, r_hi), key = min (T << 20 | r).
 // scratch: reach_scratch_bytes() for the same (p, m, R = r_hi - r_lo, vmax); counter[0]

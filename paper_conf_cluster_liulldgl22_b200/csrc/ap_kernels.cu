@@ -2263,6 +2263,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
     }
 #else
     const int ncand = 0;
+    (void)ncand;
 #endif
     __syncwarp();
     // ---- phase B: one queued job per lane, all simulated in step

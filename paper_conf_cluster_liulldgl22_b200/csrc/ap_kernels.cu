@@ -1966,6 +1966,31 @@ AP_DEV_INLINE bool pool_child(const int16_t* cur, int idx, int i, int p, int P1,
   return diff;
 }
 
+// pool_child's answer without building the child: the same size test, and for a'/b'
+// the Algorithm-1 prefix compared with cur until the first difference (cand[j] = cur[j]
+// there: the moved cut is i for a', i+1 for b').
+AP_DEV_INLINE bool pool_child_valid(const int16_t* cur, int idx, int i, int p, int P1,
+                                    const int16_t* s_arg) {
+  if (cur[i + 1] - cur[i] < 2) return false;
+  int j;
+  if (idx <= 1) {
+    if (idx == 0) return true;
+    if (i - 1 < 1) return false;
+    j = i - 1;
+  } else {
+    if (i > p - 2) return false;
+    if (idx == 2) return true;
+    j = i;
+  }
+  int e = cur[j];
+  for (int jj = j; jj >= 2; --jj) {
+    const int st = s_arg[e * P1 + jj];
+    if (st != cur[jj - 1]) return true;
+    e = st;
+  }
+  return false;
+}
+
 #ifndef AP_HEUR_MINB
 #define AP_HEUR_MINB 4
 #endif
@@ -2160,7 +2185,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
           } else
 #endif
           for (int idx = 0; idx < 4; ++idx)
-            if (pool_child<CP>(cur, idx, curM, p, P1, s_arg, scr)) {
+            if (pool_child_valid(cur, idx, curM, p, P1, s_arg)) {
               valid |= 1 << idx;
               ++nj;
             }

@@ -2129,22 +2129,25 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
           valid = 1 << 6;  // no move yet: guess a lower master first
         } else {  // the children of a step were simulated: visit them in child order
           uint32_t selT = 0xffffffffu;
-          int sel = -1, selM = 0;
+          int sel = -1, selM = 0, bidx = -1;
           for (int idx = 0; idx < 4; ++idx) {
             if (!((valid >> idx) & 1)) continue;
             ++nsims;
             const uint32_t Tc = s_chT[w][lane][idx];
             const int Mc = s_chM[w][lane][idx];
-            if (Tc < bestT) {
+            if (Tc < bestT) {  // first visited minimum; built once, below
               bestT = Tc;
-              pool_child<CP>(cur, idx, curM, p, P1, s_arg, scr);
-              copy_cuts<CP>(best, scr, P);
+              bidx = idx;
             }
             if (Mc <= curM && Tc < selT) {
               selT = Tc;
               selM = Mc;
               sel = idx;
             }
+          }
+          if (bidx >= 0 && bidx != sel) {  // from the scheme before the move
+            pool_child<CP>(cur, bidx, curM, p, P1, s_arg, scr);
+            copy_cuts<CP>(best, scr, P);
           }
           if (sel < 0) {
             walk = false;  // no child qualifies
@@ -2158,6 +2161,7 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
 #endif
             pool_child<CP>(cur, sel, curM, p, P1, s_arg, scr);
             copy_cuts<CP>(cur, scr, P);
+            if (bidx == sel) copy_cuts<CP>(best, scr, P);
             valid = (selM == curM) ? (1 << 6) : 0;  // after a same-master move guess lower
             curM = selM;
           }

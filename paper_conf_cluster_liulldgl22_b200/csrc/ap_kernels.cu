@@ -2159,9 +2159,8 @@ __global__ void __launch_bounds__(hpool::NT, AP_HEUR_MINB) k_heur_pool(HeurArgs 
               for (int idx = 0; idx < 4; ++idx) su = su && s_spM[w][lane][idx] != -2;
             }
 #endif
-            pool_child<CP>(cur, sel, curM, p, P1, s_arg, scr);
-            copy_cuts<CP>(cur, scr, P);
-            if (bidx == sel) copy_cuts<CP>(best, scr, P);
+            pool_child<CP>(cur, sel, curM, p, P1, s_arg, cur);  // in place
+            if (bidx == sel) copy_cuts<CP>(best, cur, P);
             valid = (selM == curM) ? (1 << 6) : 0;  // after a same-master move guess lower
             curM = selM;
           }
